@@ -1,0 +1,223 @@
+/*
+ * include/pf.h — C ABI of libpf_b200.so, the B200 (sm_100a) hot path of the
+ * fully distributed particle filter of Chitchian, van Amesfoort, Simonetto,
+ * Keviczky, Sips, "Adapting Particle Filter Algorithms to Many-Core
+ * Architectures", IPDPS 2013 (/root/reference/PAPER.md; "PAPER.md:16" = PDF
+ * page 4).  Readings R1–R20 and the fp32 contract F1–F11 are
+ * in DESIGN.md §3–§4.
+ *
+ * Conventions (all functions):
+ *  - Return pf_status: PF_OK (0) or a negative code.  No exceptions, no
+ *    printing.  CUDA errors are sticky on the handle (pf_last_error) and are
+ *    returned by every later call until pf_destroy.
+ *  - Device buffers (pf_buffers) are allocated and owned by the CALLER (the
+ *    Python layer uses torch), sized by pf_query_sizes, 256-byte aligned, and
+ *    must outlive the handle.  The caller owns the cudaStream_t.  The handle
+ *    owns only host metadata and small pinned staging memory.
+ *  - "host" pointers are ordinary CPU memory; "device" pointers are CUDA
+ *    device memory of the handle's device.  Work is stream-ordered on the
+ *    handle's stream; only pf_estimate / pf_get_particles / the debug hooks
+ *    synchronize it.
+ *  - A handle is used by one host thread at a time.
+ *  - Layouts: particle state is SoA, float32 [d][M_local] (row c holds state
+ *    component c of every local particle; d = n_joints + 4, components
+ *    theta_0..theta_{n_j-1}, x, y, v_x, v_y — PAPER.md:22 §VII-A); local
+ *    particle column = n_local * m + i for sub-filter n_local, slot i; the
+ *    log-weight ("logw", reading R7) is float32 [M_local].
+ */
+#ifndef PF_H
+#define PF_H
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+  PF_OK = 0,
+  PF_EINVAL = -1,        /* invalid argument / configuration                 */
+  PF_ENOMEM = -2,        /* host allocation failed                           */
+  PF_ECUDA = -3,         /* CUDA error (sticky)                              */
+  PF_ESTATE = -5,        /* call not valid in the handle's state             */
+  PF_EUNSUPPORTED = -6   /* (n_joints, m) combination not compiled           */
+} pf_status;
+
+/* Exchange scheme X (PAPER.md:18 Table I; :16 Fig.1; :20 §VI-E). */
+typedef enum { PF_TOPO_NONE = 0, PF_TOPO_RING = 1, PF_TOPO_TORUS2D = 2 } pf_topology;
+/* Resampler (PAPER.md:18 §IV; :20–22 §VI-F). */
+typedef enum { PF_RESAMPLE_RWS = 0, PF_RESAMPLE_VOSE = 1 } pf_resampler;
+/* Model hooks (the paper separates "generic particle filtering from
+ * model-specific routines", §I).  The robotic arm of
+ * PAPER.md:22–24 §VII-A with h(x) of reading R14; compiled for
+ * n_joints in {2, 5, 28}. */
+typedef enum { PF_MODEL_ARM_PLANAR = 0 } pf_model_id;
+
+/* pf_config.flags */
+#define PF_DEVICE_INPUTS 1u   /* pf_step's z / u are device pointers         */
+
+typedef struct {
+  int32_t model;            /* pf_model_id                                           */
+  int32_t n_joints;         /* joints incl. base rotation; d = n_joints + 4          */
+  float arm_length;         /* L (m); link length L / n_joints (R16)                 */
+  float h_s;                /* sampling time (s) (R16)                               */
+  float sigma_theta;        /* process noise std, joint angles (R15)                 */
+  float sigma_pos;          /* process noise std, object x, y                        */
+  float sigma_vel;          /* process noise std, object v_x, v_y                    */
+  float sigma_cam;          /* measurement noise std, camera (x_C, y_C)              */
+  float sigma_theta_meas;   /* measurement noise std, joint sensors                  */
+} pf_model_params;
+
+/* Table I: m, N, X, t; plus resampler, RNG seed and the shard
+ * of this process.  Sharding: ring — rank r owns global
+ * sub-filters [r N/W, (r+1) N/W); torus — rank r owns rows
+ * [r R/W, (r+1) R/W) of the R x C grid. */
+typedef struct {
+  int32_t m;                /* particles per sub-filter, power of two in [32, 1024]  */
+  int64_t n_filters;        /* N, GLOBAL number of sub-filters                       */
+  int32_t t;                /* particles per exchange per neighbour; deg*t < m (R19) */
+  int32_t topo;             /* pf_topology                                           */
+  int32_t torus_rows;       /* 0 = default R = 2^floor(log2(N)/2) (R4)               */
+  int32_t torus_cols;       /* 0 = default N / R                                     */
+  int32_t resampler;        /* pf_resampler                                          */
+  uint64_t seed;            /* Philox key = (seed & 0xffffffff, seed >> 32) (R12)    */
+  int32_t rank;             /* shard index in [0, world)                             */
+  int32_t world;            /* number of shards (processes / GPUs), >= 1             */
+  uint32_t flags;           /* PF_DEVICE_INPUTS                                      */
+} pf_config;
+
+/* Bytes of each caller-owned device buffer. */
+typedef struct {
+  uint64_t state;    /* float [d][M_local]                                          */
+  uint64_t logw;     /* float [M_local]                                             */
+  uint64_t mailbox;  /* float [2][n_ext][max(t,1)][d+2]: exchange mailbox, see below */
+  uint64_t scratch;  /* keys, counters, estimate record, step inputs                */
+} pf_sizes;
+
+typedef struct {
+  void* state;
+  void* logw;
+  void* mailbox;
+  void* scratch;
+} pf_buffers;
+
+/* Shard geometry (multi-rank plumbing).  Mailbox entry (d+2 floats) =
+ * [logw, global particle index (uint32 bits), x_0..x_{d-1}]; mailbox parity
+ * k&1 holds the best t of every local sub-filter after step k at rows
+ * [0, n_local), and rows [n_local, n_ext) are halo rows the caller fills
+ * with neighbour ranks' entries before step k+1: ring — row n_local holds
+ * global sub-filter (g0-1) mod N, row n_local+1 holds (g0+n_local) mod N;
+ * torus — rows n_local + c hold grid row (r0-1) mod R, rows
+ * n_local + C + c hold grid row (r1) mod R (c = column). */
+typedef struct {
+  int64_t g0;            /* first global sub-filter of this shard                  */
+  int64_t n_local;       /* local sub-filters                                      */
+  int64_t n_ext;         /* n_local + halo rows                                    */
+  int64_t torus_rows;    /* R (torus) or 0                                         */
+  int64_t torus_cols;    /* C (torus) or 0                                         */
+  int32_t entry_floats;  /* d + 2                                                  */
+  int32_t t;             /* entries per sub-filter row (max(t, 1))                 */
+  int32_t d;             /* state dimension                                        */
+  int32_t record_floats; /* 4 + d                                                  */
+} pf_shard;
+
+typedef struct pf_handle pf_handle;
+
+/* Sizes of the caller-owned buffers for (cfg, model).  PF_EINVAL on an
+ * invalid configuration (same checks as pf_init). */
+pf_status pf_query_sizes(const pf_config* cfg, const pf_model_params* model, pf_sizes* out);
+
+/* Create a handle on the current CUDA device and draw the initial particle
+ * set X_0 ~ N(mu0, diag(sigma0^2)) (implicit input of Algorithm 2, PAPER.md:16;
+ * F11, Philox stream 2).  mu0, sigma0: host float[d].  cuda_stream: a
+ * cudaStream_t (NULL = legacy default stream).  Validation (PF_EINVAL): m a
+ * power of two in [32, 1024]; deg*t < m; N % world == 0 (ring) or
+ * R % world == 0 and R*C == N (torus); N*m per shard <= 2^31; global N*m <= 2^32;
+ * 0 <= rank < world; unsupported n_joints -> PF_EUNSUPPORTED. */
+pf_status pf_init(const pf_config* cfg, const pf_model_params* model, const pf_buffers* buffers,
+                  void* cuda_stream, const float* mu0, const float* sigma0, pf_handle** out);
+
+/* One time step k = (last step) + 1 of Algorithm 2: exchange
+ * with the neighbours' best t of step k-1 (l.10–14), normalise + resample
+ * locally (l.15–19), sample + weight (l.3–6), local/global estimate (l.8–9).
+ * z_k: float[n_joints + 2] = (x_C, y_C, theta_hat_0..), u_{k-1}:
+ * float[n_joints].  Host pointers (copied to the device
+ * inside the call's stream work) unless PF_DEVICE_INPUTS.  Asynchronous.
+ * With world > 1 the caller must have filled the halo rows of mailbox
+ * parity (k-1)&1 (see pf_shard) and, after the step, reduce the per-rank
+ * records (pf_reduce_records) for a global estimate. */
+pf_status pf_step(pf_handle* h, const float* z_k, const float* u_km1);
+
+/* T consecutive steps with device-resident inputs zs [T][n_joints+2] and
+ * us [T][n_joints] (device), writing each step's estimate record
+ * (4 + d floats, layout of pf_record_ptr) to est [T][4+d] (device, nullable).
+ * world == 1 only (PF_ESTATE otherwise).  Asynchronous (T back-to-back
+ * launches on the handle's stream, no host synchronization). */
+pf_status pf_step_batch(pf_handle* h, int32_t T, const float* zs, const float* us, float* est);
+
+/* The global estimate of the last step: the particle with the highest
+ * weight (PAPER.md:16 §IV; :20 §VI-D; R6).  Synchronizes the stream.
+ * x_hat: host float[d]; logw, idx (global particle index): host, nullable.
+ * PF_ESTATE before the first step. */
+pf_status pf_estimate(pf_handle* h, float* x_hat, float* logw, int64_t* idx);
+
+/* Device pointer to this shard's estimate record of the last step:
+ * float[4 + d] = [key lo (u32 bits), key hi (u32 bits), logw, reserved, x[d]]
+ * with key = (ordered(logw) << 32) | (0xffffffff - global index). */
+pf_status pf_record_ptr(pf_handle* h, float** record_dev, int32_t* record_floats);
+
+/* Global estimate from `count` records (device, [count][4+d], e.g. an
+ * all-gather of every rank's record): picks the maximal key (exact,
+ * order-free) and makes it this handle's estimate.  Asynchronous. */
+pf_status pf_reduce_records(pf_handle* h, const float* records_dev, int32_t count);
+
+/* Shard geometry and mailbox layout for halo exchange. */
+pf_status pf_get_shard(const pf_handle* h, pf_shard* out);
+
+/* Checkpoint: copy the weighted particle set of the last step (state
+ * [d][M_local], logw [M_local], host) and its step index (step 0 = prior,
+ * logw undefined).  Synchronizes. */
+pf_status pf_get_particles(pf_handle* h, float* state_host, float* logw_host, int64_t* step);
+/* Resume: load a weighted particle set as the result of step `step` >= 1
+ * (host pointers), republish its best t to the mailbox and its estimate.
+ * With the counter-based RNG, resuming is bit-exact.  Synchronizes. */
+pf_status pf_set_particles(pf_handle* h, const float* state_host, const float* logw_host, int64_t step);
+
+/* ---- test hooks: the same device code on isolated phases.  They clobber
+ * the handle's particles, mailbox and estimate.  world == 1 only. ---- */
+
+/* Sample + weight (a1–a3) every particle of state_in [d][M] (host) with no
+ * resampling, Philox counter (p, k, 0, j) (R13): state_out [d][M],
+ * logw_out [M] (host). */
+pf_status pf_debug_sample_weight(pf_handle* h, const float* state_in, const float* z_k,
+                                 const float* u_km1, int64_t k, float* state_out, float* logw_out);
+
+/* Resampling (a8) of integer weights q [N][m] (host, each row with
+ * sum > 0 and sum <= 2^32) with explicit uniforms ua, ub [N][m] (host):
+ * ancestors [N][m] (host).  Vose only: prob [N][m] (uint64, units of the
+ * row sum) and alias [N][m] (host, nullable) of the alias table (R10). */
+pf_status pf_debug_resample(pf_handle* h, const uint32_t* q, const uint32_t* ua, const uint32_t* ub,
+                            int32_t* ancestors, uint64_t* prob, int32_t* alias);
+
+/* Exchange (a6) of log-weights logw [N][m] (host): src [N][m] (host) = the
+ * global index of the particle each slot holds after the exchange (R2–R5). */
+pf_status pf_debug_exchange(pf_handle* h, const float* logw, int64_t* src);
+
+/* Exchange sources and ancestors of the last pf_step (host, [M_local] each,
+ * nullable); recorded only when PF_TRACE was enabled with pf_set_trace. */
+pf_status pf_set_trace(pf_handle* h, int32_t enable);
+pf_status pf_get_trace(pf_handle* h, int64_t* src, int32_t* ancestors);
+
+/* Release host metadata; NULL-safe.  Does not free caller buffers. */
+pf_status pf_destroy(pf_handle* h);
+
+const char* pf_strerror(pf_status s);
+pf_status pf_last_error(const pf_handle* h);
+
+/* Compiled configurations: writes up to `cap` (n_joints, m) pairs. */
+int32_t pf_supported(int32_t* n_joints, int32_t* m, int32_t cap);
+
+#ifdef __cplusplus
+}
+#endif
+#endif

@@ -1,0 +1,626 @@
+// pf_runtime.cu — host runtime behind the C ABI of include/pf.h.
+//
+// Owns host metadata only: configuration validation, shard geometry, the
+// scratch carve-up of the caller's buffers, the kernel table lookup, the
+// per-step launch parameters, and small pinned staging for step inputs.
+// Every computation of the path runs in the kernels of pf_kernels.cuh.
+#include <cuda_runtime.h>
+
+#include <cstdint>
+#include <cstdlib>
+#include <cstring>
+#include <new>
+
+#include "../../include/pf.h"
+#include "pf_kernels.cuh"
+#include "pf_registry.h"
+
+using pf::u64;
+
+namespace {
+
+constexpr int kMaxNJ = 28;
+constexpr int kStageSlots = 8;
+
+// scratch layout (bytes)
+constexpr size_t kOffKeys = 0;        // u64[2]
+constexpr size_t kOffCounter = 16;    // u32
+constexpr size_t kOffRecord = 64;     // float[4 + d]  (d <= 32 -> 144 B)
+constexpr size_t kOffInputs = 256;    // float[64]: z at 0, u at 32
+constexpr size_t kOffMu0 = 512;       // float[64]
+constexpr size_t kOffSigma0 = 768;    // float[64]
+constexpr size_t kScratchBytes = 1024;
+
+const pf::KernelEntry* find_entry(int nj, int m, int res) {
+  const pf::KernelEntry* tables[] = {pf::kEntriesNJ2, pf::kEntriesNJ5, pf::kEntriesNJ28};
+  for (const pf::KernelEntry* t : tables)
+    for (int i = 0; i < pf::kNumEntriesPerNJ; ++i)
+      if (t[i].nj == nj && t[i].m == m && t[i].res == res) return &t[i];
+  return nullptr;
+}
+
+struct Geometry {
+  int nj, d, m, deg, tt, E;
+  long long N, R, C, n_local, g0, n_ext, M_local;
+};
+
+pf_status validate(const pf_config* cfg, const pf_model_params* mp, Geometry* g) {
+  if (!cfg || !mp) return PF_EINVAL;
+  if (mp->model != PF_MODEL_ARM_PLANAR || mp->n_joints < 1) return PF_EINVAL;
+  if (!(mp->sigma_cam > 0.0f) || !(mp->sigma_theta_meas > 0.0f) || !(mp->sigma_theta >= 0.0f) ||
+      !(mp->sigma_pos >= 0.0f) || !(mp->sigma_vel >= 0.0f))
+    return PF_EINVAL;
+  const int m = cfg->m;
+  if (m < 32 || m > 1024 || (m & (m - 1)) != 0) return PF_EINVAL;
+  if (cfg->n_filters < 1 || cfg->t < 0 || cfg->world < 1 || cfg->rank < 0 || cfg->rank >= cfg->world)
+    return PF_EINVAL;
+  if (cfg->resampler != PF_RESAMPLE_RWS && cfg->resampler != PF_RESAMPLE_VOSE) return PF_EINVAL;
+  if (cfg->topo != PF_TOPO_NONE && cfg->topo != PF_TOPO_RING && cfg->topo != PF_TOPO_TORUS2D) return PF_EINVAL;
+  if (!find_entry(mp->n_joints, m, cfg->resampler)) return PF_EUNSUPPORTED;
+  g->nj = mp->n_joints;
+  g->d = mp->n_joints + 4;
+  g->m = m;
+  g->N = cfg->n_filters;
+  g->deg = cfg->topo == PF_TOPO_RING ? 2 : cfg->topo == PF_TOPO_TORUS2D ? 4 : 0;
+  if (static_cast<long long>(g->deg) * cfg->t >= m && g->deg * cfg->t > 0) return PF_EINVAL;   // R19
+  if (g->deg * cfg->t > 128) return PF_EINVAL;
+  g->tt = cfg->t > 0 ? cfg->t : 1;
+  g->E = g->d + 2;
+  g->R = g->C = 0;
+  const long long W = cfg->world;
+  if (cfg->topo == PF_TOPO_TORUS2D) {
+    long long R = cfg->torus_rows, C = cfg->torus_cols;
+    if (R <= 0 || C <= 0) {
+      int lg = 0;
+      while ((1ll << (lg + 1)) <= g->N) ++lg;
+      R = 1ll << (lg / 2);
+      C = g->N / R;
+    }
+    if (R * C != g->N || R % W != 0) return PF_EINVAL;
+    g->R = R;
+    g->C = C;
+    const long long rows = R / W;
+    g->n_local = rows * C;
+    g->g0 = cfg->rank * rows * C;
+    g->n_ext = g->n_local + (W > 1 ? 2 * C : 0);
+  } else {
+    if (g->N % W != 0) return PF_EINVAL;
+    g->n_local = g->N / W;
+    g->g0 = cfg->rank * g->n_local;
+    g->n_ext = g->n_local + ((W > 1 && cfg->topo == PF_TOPO_RING) ? 2 : 0);
+  }
+  g->M_local = g->n_local * m;
+  if (g->M_local > (1ll << 31) || g->N * m > (1ll << 32)) return PF_EINVAL;
+  return PF_OK;
+}
+
+}  // namespace
+
+struct pf_handle {
+  pf_config cfg;
+  pf_model_params mp;
+  Geometry g;
+  pf::ArmConsts mc;
+  float* state;
+  float* logw;
+  float* mailbox;
+  unsigned char* scratch;
+  cudaStream_t stream;
+  long long step;
+  const pf::KernelEntry* ke;
+  int grid;
+  pf_status err;
+  float* pinned;                 // [kStageSlots][64]
+  cudaEvent_t stage_ev[kStageSlots];
+  int stage_next;
+  bool trace;
+  long long* d_src;
+  int* d_anc;
+  float* d_reduce_tmp;
+};
+
+namespace {
+
+pf_status sticky(pf_handle* h, cudaError_t e) {
+  if (e != cudaSuccess && h->err == PF_OK) h->err = PF_ECUDA;
+  return e == cudaSuccess ? h->err : PF_ECUDA;
+}
+
+u64* keys(pf_handle* h) { return reinterpret_cast<u64*>(h->scratch + kOffKeys); }
+float* record(pf_handle* h) { return reinterpret_cast<float*>(h->scratch + kOffRecord); }
+float* inputs(pf_handle* h) { return reinterpret_cast<float*>(h->scratch + kOffInputs); }
+
+float* mailbox_parity(pf_handle* h, long long k) {
+  return h->mailbox + (k & 1) * h->g.n_ext * h->g.tt * h->g.E;
+}
+
+pf::StepParams base_params(pf_handle* h, long long k, int mode) {
+  pf::StepParams p;
+  std::memset(&p, 0, sizeof(p));
+  p.mc = h->mc;
+  p.state = h->state;
+  p.logw = h->logw;
+  p.stride = h->g.M_local;
+  p.mb_prev = mailbox_parity(h, k - 1);
+  p.mb_cur = mailbox_parity(h, k);
+  p.z = inputs(h);
+  p.u = inputs(h) + 32;
+  p.key_cur = keys(h) + (k & 1);
+  p.key_next = keys(h) + ((k + 1) & 1);
+  p.counter = reinterpret_cast<unsigned int*>(h->scratch + kOffCounter);
+  p.record = record(h);
+  p.est_out = nullptr;
+  p.dbg_src = nullptr;
+  p.dbg_anc = nullptr;
+  p.n_local = h->g.n_local;
+  p.g0 = h->g.g0;
+  p.n_global = h->g.N;
+  p.R = h->g.R;
+  p.C = h->g.C;
+  p.t = h->cfg.t;
+  p.tt = h->g.tt;
+  p.topo = h->cfg.topo;
+  p.deg = h->g.deg;
+  p.key0 = static_cast<uint32_t>(h->cfg.seed);
+  p.key1 = static_cast<uint32_t>(h->cfg.seed >> 32);
+  p.k = static_cast<uint32_t>(k);
+  p.mode = mode;
+  p.first = (k == 1) ? 1 : 0;
+  return p;
+}
+
+// Copy z (n_j+2) and u (n_j) host -> device inputs through a pinned slot.
+pf_status stage_inputs(pf_handle* h, const float* z, const float* u) {
+  const int nj = h->g.nj;
+  float* slot = h->pinned + h->stage_next * 64;
+  cudaError_t e = cudaEventSynchronize(h->stage_ev[h->stage_next]);
+  if (e != cudaSuccess) return sticky(h, e);
+  std::memcpy(slot, z, sizeof(float) * (nj + 2));
+  std::memcpy(slot + 32, u, sizeof(float) * nj);
+  e = cudaMemcpyAsync(inputs(h), slot, sizeof(float) * (32 + nj), cudaMemcpyHostToDevice, h->stream);
+  if (e == cudaSuccess) e = cudaEventRecord(h->stage_ev[h->stage_next], h->stream);
+  h->stage_next = (h->stage_next + 1) % kStageSlots;
+  return sticky(h, e);
+}
+
+pf_status launch(pf_handle* h, const pf::StepParams& p) {
+  return sticky(h, h->ke->launch(p, h->grid, h->stream));
+}
+
+__global__ void pf_init_kernel(float* state, float* logw, long long stride, long long M_local, uint32_t p0, int d,
+                               const float* mu0, const float* s0, uint32_t key0, uint32_t key1) {
+  // F11: x_c = fma(sigma0_c, xi_c, mu0_c); pair q of particle p from words
+  // 2(q&1), 2(q&1)+1 of Philox (p, 0, 2, q>>1) (R13, stream 2 = init).
+  for (long long col = blockIdx.x * static_cast<long long>(blockDim.x) + threadIdx.x; col < M_local;
+       col += static_cast<long long>(gridDim.x) * blockDim.x) {
+    const uint32_t p = p0 + static_cast<uint32_t>(col);
+    pf::u32x4 blk{0, 0, 0, 0};
+    for (int q = 0; q < (d + 1) / 2; ++q) {
+      if ((q & 1) == 0) blk = pf::philox4x32_10(p, 0u, 2u, static_cast<uint32_t>(q >> 1), key0, key1);
+      const uint32_t x0 = (q & 1) ? blk.z : blk.x;
+      const uint32_t x1 = (q & 1) ? blk.w : blk.y;
+      float z0, z1;
+      pf::normal_pair(x0, x1, z0, z1);
+      const int c = 2 * q;
+      state[c * stride + col] = __fmaf_rn(s0[c], z0, mu0[c]);
+      if (c + 1 < d) state[(c + 1) * stride + col] = __fmaf_rn(s0[c + 1], z1, mu0[c + 1]);
+    }
+    logw[col] = 0.0f;
+  }
+}
+
+// Pick the record with the maximal key among `count` (exact, order-free).
+__global__ void pf_reduce_records_kernel(const float* recs, int count, int rec_floats, float* out) {
+  const int lane = threadIdx.x;
+  u64 best = 0ull;
+  int bi = 0;
+  for (int i = lane; i < count; i += 32) {
+    const u64 k = static_cast<u64>(__float_as_uint(recs[i * rec_floats])) |
+                  (static_cast<u64>(__float_as_uint(recs[i * rec_floats + 1])) << 32);
+    if (k > best) {
+      best = k;
+      bi = i;
+    }
+  }
+  const uint32_t hi = __reduce_max_sync(0xFFFFFFFFu, static_cast<uint32_t>(best >> 32));
+  const uint32_t lo =
+      __reduce_max_sync(0xFFFFFFFFu, static_cast<uint32_t>(best >> 32) == hi ? static_cast<uint32_t>(best) : 0u);
+  const u64 win = (static_cast<u64>(hi) << 32) | lo;
+  const unsigned mask = __ballot_sync(0xFFFFFFFFu, best == win);
+  const int src_lane = __ffs(mask) - 1;
+  const int src = __shfl_sync(0xFFFFFFFFu, bi, src_lane);
+  for (int c = lane; c < rec_floats; c += 32) out[c] = recs[src * rec_floats + c];
+}
+
+template <int M, int RES>
+cudaError_t launch_resample_debug(const uint32_t* q, const uint32_t* ua, const uint32_t* ub, int* anc, u64* prob,
+                                  int* alias, long long N, cudaStream_t s) {
+  const int grid = static_cast<int>(N < 4096 ? N : 4096);
+  pf::pf_resample_debug_kernel<M, RES><<<grid, M, 0, s>>>(q, ua, ub, anc, prob, alias, N);
+  return cudaGetLastError();
+}
+
+cudaError_t resample_debug_dispatch(int m, int res, const uint32_t* q, const uint32_t* ua, const uint32_t* ub,
+                                    int* anc, u64* prob, int* alias, long long N, cudaStream_t s) {
+#define PF_RD(MM)                                                                    \
+  case MM:                                                                           \
+    return res ? launch_resample_debug<MM, 1>(q, ua, ub, anc, prob, alias, N, s) \
+               : launch_resample_debug<MM, 0>(q, ua, ub, anc, prob, alias, N, s);
+  switch (m) {
+    PF_RD(32)
+    PF_RD(64)
+    PF_RD(128)
+    PF_RD(256)
+    PF_RD(512)
+    PF_RD(1024)
+    default:
+      return cudaErrorInvalidValue;
+  }
+#undef PF_RD
+}
+
+template <typename T>
+struct DevBuf {
+  T* p = nullptr;
+  cudaError_t alloc(size_t n) { return cudaMalloc(&p, sizeof(T) * (n ? n : 1)); }
+  ~DevBuf() {
+    if (p) cudaFree(p);
+  }
+};
+
+}  // namespace
+
+namespace pf {
+const int kNumEntriesPerNJ = 12;
+}
+
+extern "C" {
+
+pf_status pf_query_sizes(const pf_config* cfg, const pf_model_params* model, pf_sizes* out) {
+  Geometry g;
+  const pf_status s = validate(cfg, model, &g);
+  if (s != PF_OK || !out) return s != PF_OK ? s : PF_EINVAL;
+  out->state = sizeof(float) * g.d * g.M_local;
+  out->logw = sizeof(float) * g.M_local;
+  out->mailbox = sizeof(float) * 2 * g.n_ext * g.tt * g.E;
+  out->scratch = kScratchBytes;
+  return PF_OK;
+}
+
+pf_status pf_init(const pf_config* cfg, const pf_model_params* model, const pf_buffers* buffers,
+                  void* cuda_stream, const float* mu0, const float* sigma0, pf_handle** out) {
+  if (!out || !buffers || !mu0 || !sigma0) return PF_EINVAL;
+  *out = nullptr;
+  Geometry g;
+  pf_status s = validate(cfg, model, &g);
+  if (s != PF_OK) return s;
+  if (!buffers->state || !buffers->logw || !buffers->mailbox || !buffers->scratch) return PF_EINVAL;
+  pf_handle* h = new (std::nothrow) pf_handle();
+  if (!h) return PF_ENOMEM;
+  h->cfg = *cfg;
+  h->mp = *model;
+  h->g = g;
+  // F9/F10 model constants: fp32 operations, exactly as the contract states
+  h->mc.lj = model->arm_length / static_cast<float>(model->n_joints);
+  h->mc.hs = model->h_s;
+  h->mc.s_th = model->sigma_theta;
+  h->mc.s_pos = model->sigma_pos;
+  h->mc.s_vel = model->sigma_vel;
+  h->mc.inv_cam = 1.0f / model->sigma_cam;
+  h->mc.inv_thm = 1.0f / model->sigma_theta_meas;
+  h->state = static_cast<float*>(buffers->state);
+  h->logw = static_cast<float*>(buffers->logw);
+  h->mailbox = static_cast<float*>(buffers->mailbox);
+  h->scratch = static_cast<unsigned char*>(buffers->scratch);
+  h->stream = static_cast<cudaStream_t>(cuda_stream);
+  h->step = 0;
+  h->ke = find_entry(g.nj, g.m, cfg->resampler);
+  h->err = PF_OK;
+  int dev = 0, sms = 0, bps = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e == cudaSuccess) e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  if (e == cudaSuccess) e = h->ke->prepare(&bps);
+  if (e == cudaSuccess && bps < 1) e = cudaErrorInvalidConfiguration;
+  if (e == cudaSuccess) e = cudaMallocHost(reinterpret_cast<void**>(&h->pinned), sizeof(float) * 64 * kStageSlots);
+  for (int i = 0; i < kStageSlots && e == cudaSuccess; ++i)
+    e = cudaEventCreateWithFlags(&h->stage_ev[i], cudaEventDisableTiming);
+  if (e != cudaSuccess) {
+    pf_destroy(h);
+    return PF_ECUDA;
+  }
+  const long long grid = static_cast<long long>(bps) * sms;
+  h->grid = static_cast<int>(grid < g.n_local ? grid : g.n_local);
+  // scratch: zero keys / counter; prior parameters
+  float prior[128];
+  std::memset(prior, 0, sizeof(prior));
+  std::memcpy(prior, mu0, sizeof(float) * g.d);
+  std::memcpy(prior + 64, sigma0, sizeof(float) * g.d);
+  e = cudaMemsetAsync(h->scratch, 0, kScratchBytes, h->stream);
+  if (e == cudaSuccess)
+    e = cudaMemcpyAsync(h->scratch + kOffMu0, prior, sizeof(prior), cudaMemcpyHostToDevice, h->stream);
+  if (e == cudaSuccess) e = cudaMemsetAsync(h->mailbox, 0, sizeof(float) * 2 * g.n_ext * g.tt * g.E, h->stream);
+  if (e == cudaSuccess) {
+    const long long blocks = (g.M_local + 255) / 256;
+    pf_init_kernel<<<static_cast<int>(blocks < 8 * sms ? blocks : 8 * sms), 256, 0, h->stream>>>(
+        h->state, h->logw, g.M_local, g.M_local, static_cast<uint32_t>(g.g0 * g.m), g.d,
+        reinterpret_cast<const float*>(h->scratch + kOffMu0), reinterpret_cast<const float*>(h->scratch + kOffSigma0),
+        static_cast<uint32_t>(cfg->seed), static_cast<uint32_t>(cfg->seed >> 32));
+    e = cudaGetLastError();
+  }
+  // the prior copy reads a stack buffer: finish before returning
+  if (e == cudaSuccess) e = cudaStreamSynchronize(h->stream);
+  if (e != cudaSuccess) {
+    pf_destroy(h);
+    return PF_ECUDA;
+  }
+  *out = h;
+  return PF_OK;
+}
+
+pf_status pf_step(pf_handle* h, const float* z_k, const float* u_km1) {
+  if (!h || !z_k || !u_km1) return PF_EINVAL;
+  if (h->err != PF_OK) return h->err;
+  const long long k = h->step + 1;
+  pf::StepParams p = base_params(h, k, pf::MODE_STEP);
+  if (h->cfg.flags & PF_DEVICE_INPUTS) {
+    p.z = z_k;
+    p.u = u_km1;
+  } else {
+    const pf_status s = stage_inputs(h, z_k, u_km1);
+    if (s != PF_OK) return s;
+  }
+  if (h->trace) {
+    p.dbg_src = h->d_src;
+    p.dbg_anc = h->d_anc;
+  }
+  const pf_status s = launch(h, p);
+  if (s == PF_OK) h->step = k;
+  return s;
+}
+
+pf_status pf_step_batch(pf_handle* h, int32_t T, const float* zs, const float* us, float* est) {
+  if (!h || T < 0 || (T > 0 && (!zs || !us))) return PF_EINVAL;
+  if (h->err != PF_OK) return h->err;
+  if (h->cfg.world != 1) return PF_ESTATE;
+  const int nj = h->g.nj;
+  for (int32_t s = 0; s < T; ++s) {
+    const long long k = h->step + 1;
+    pf::StepParams p = base_params(h, k, pf::MODE_STEP);
+    p.z = zs + static_cast<long long>(s) * (nj + 2);
+    p.u = us + static_cast<long long>(s) * nj;
+    p.est_out = est ? est + static_cast<long long>(s) * (4 + h->g.d) : nullptr;
+    if (h->trace) {
+      p.dbg_src = h->d_src;
+      p.dbg_anc = h->d_anc;
+    }
+    const pf_status st = launch(h, p);
+    if (st != PF_OK) return st;
+    h->step = k;
+  }
+  return PF_OK;
+}
+
+pf_status pf_estimate(pf_handle* h, float* x_hat, float* logw, int64_t* idx) {
+  if (!h || !x_hat) return PF_EINVAL;
+  if (h->err != PF_OK) return h->err;
+  if (h->step < 1) return PF_ESTATE;
+  float rec[4 + 32 + 4];
+  cudaError_t e = cudaMemcpyAsync(rec, record(h), sizeof(float) * (4 + h->g.d), cudaMemcpyDeviceToHost, h->stream);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(h->stream);
+  if (e != cudaSuccess) return sticky(h, e);
+  uint32_t lo;
+  std::memcpy(&lo, &rec[0], 4);
+  std::memcpy(x_hat, rec + 4, sizeof(float) * h->g.d);
+  if (logw) *logw = rec[2];
+  if (idx) *idx = static_cast<int64_t>(0xFFFFFFFFu - lo);
+  return PF_OK;
+}
+
+pf_status pf_record_ptr(pf_handle* h, float** record_dev, int32_t* record_floats) {
+  if (!h || !record_dev) return PF_EINVAL;
+  *record_dev = record(h);
+  if (record_floats) *record_floats = 4 + h->g.d;
+  return h->err;
+}
+
+pf_status pf_reduce_records(pf_handle* h, const float* records_dev, int32_t count) {
+  if (!h || !records_dev || count < 1) return PF_EINVAL;
+  if (h->err != PF_OK) return h->err;
+  pf_reduce_records_kernel<<<1, 32, 0, h->stream>>>(records_dev, count, 4 + h->g.d, record(h));
+  return sticky(h, cudaGetLastError());
+}
+
+pf_status pf_get_shard(const pf_handle* h, pf_shard* out) {
+  if (!h || !out) return PF_EINVAL;
+  out->g0 = h->g.g0;
+  out->n_local = h->g.n_local;
+  out->n_ext = h->g.n_ext;
+  out->torus_rows = h->g.R;
+  out->torus_cols = h->g.C;
+  out->entry_floats = h->g.E;
+  out->t = h->g.tt;
+  out->d = h->g.d;
+  out->record_floats = 4 + h->g.d;
+  return PF_OK;
+}
+
+pf_status pf_get_particles(pf_handle* h, float* state_host, float* logw_host, int64_t* step) {
+  if (!h || !state_host) return PF_EINVAL;
+  if (h->err != PF_OK) return h->err;
+  cudaError_t e = cudaStreamSynchronize(h->stream);
+  if (e == cudaSuccess)
+    e = cudaMemcpy(state_host, h->state, sizeof(float) * h->g.d * h->g.M_local, cudaMemcpyDeviceToHost);
+  if (e == cudaSuccess && logw_host)
+    e = cudaMemcpy(logw_host, h->logw, sizeof(float) * h->g.M_local, cudaMemcpyDeviceToHost);
+  if (step) *step = h->step;
+  return sticky(h, e);
+}
+
+static pf_status publish(pf_handle* h, long long step) {
+  cudaError_t e = cudaMemsetAsync(keys(h), 0, 2 * sizeof(u64), h->stream);
+  if (e != cudaSuccess) return sticky(h, e);
+  pf::StepParams p = base_params(h, step, pf::MODE_PUBLISH);
+  return launch(h, p);
+}
+
+pf_status pf_set_particles(pf_handle* h, const float* state_host, const float* logw_host, int64_t step) {
+  if (!h || !state_host || !logw_host || step < 1) return PF_EINVAL;
+  if (h->err != PF_OK) return h->err;
+  cudaError_t e = cudaStreamSynchronize(h->stream);
+  if (e == cudaSuccess)
+    e = cudaMemcpy(h->state, state_host, sizeof(float) * h->g.d * h->g.M_local, cudaMemcpyHostToDevice);
+  if (e == cudaSuccess) e = cudaMemcpy(h->logw, logw_host, sizeof(float) * h->g.M_local, cudaMemcpyHostToDevice);
+  if (e != cudaSuccess) return sticky(h, e);
+  pf_status s = publish(h, step);
+  if (s != PF_OK) return s;
+  h->step = step;
+  return sticky(h, cudaStreamSynchronize(h->stream));
+}
+
+pf_status pf_debug_sample_weight(pf_handle* h, const float* state_in, const float* z_k, const float* u_km1,
+                                 int64_t k, float* state_out, float* logw_out) {
+  if (!h || !state_in || !z_k || !u_km1 || !state_out || !logw_out || k < 1) return PF_EINVAL;
+  if (h->err != PF_OK) return h->err;
+  if (h->cfg.world != 1) return PF_ESTATE;
+  cudaError_t e = cudaStreamSynchronize(h->stream);
+  if (e == cudaSuccess)
+    e = cudaMemcpy(h->state, state_in, sizeof(float) * h->g.d * h->g.M_local, cudaMemcpyHostToDevice);
+  if (e == cudaSuccess) e = cudaMemsetAsync(keys(h), 0, 2 * sizeof(u64), h->stream);
+  if (e != cudaSuccess) return sticky(h, e);
+  pf_status s = stage_inputs(h, z_k, u_km1);
+  if (s != PF_OK) return s;
+  pf::StepParams p = base_params(h, k, pf::MODE_SAMPLE);
+  s = launch(h, p);
+  if (s != PF_OK) return s;
+  h->step = k;
+  e = cudaStreamSynchronize(h->stream);
+  if (e == cudaSuccess)
+    e = cudaMemcpy(state_out, h->state, sizeof(float) * h->g.d * h->g.M_local, cudaMemcpyDeviceToHost);
+  if (e == cudaSuccess) e = cudaMemcpy(logw_out, h->logw, sizeof(float) * h->g.M_local, cudaMemcpyDeviceToHost);
+  return sticky(h, e);
+}
+
+pf_status pf_debug_resample(pf_handle* h, const uint32_t* q, const uint32_t* ua, const uint32_t* ub,
+                            int32_t* ancestors, uint64_t* prob, int32_t* alias) {
+  if (!h || !q || !ua || !ub || !ancestors) return PF_EINVAL;
+  if (h->err != PF_OK) return h->err;
+  const long long n = h->g.N * h->g.m;
+  DevBuf<uint32_t> dq, dua, dub;
+  DevBuf<int> danc, dal;
+  DevBuf<u64> dpr;
+  const bool vose = h->cfg.resampler == PF_RESAMPLE_VOSE;
+  const bool want_table = vose && prob && alias;
+  cudaError_t e = dq.alloc(n);
+  if (e == cudaSuccess) e = dua.alloc(n);
+  if (e == cudaSuccess) e = dub.alloc(n);
+  if (e == cudaSuccess) e = danc.alloc(n);
+  if (e == cudaSuccess && want_table) e = dpr.alloc(n);
+  if (e == cudaSuccess && want_table) e = dal.alloc(n);
+  if (e == cudaSuccess) e = cudaMemcpy(dq.p, q, 4 * n, cudaMemcpyHostToDevice);
+  if (e == cudaSuccess) e = cudaMemcpy(dua.p, ua, 4 * n, cudaMemcpyHostToDevice);
+  if (e == cudaSuccess) e = cudaMemcpy(dub.p, ub, 4 * n, cudaMemcpyHostToDevice);
+  if (e == cudaSuccess)
+    e = resample_debug_dispatch(h->g.m, vose ? 1 : 0, dq.p, dua.p, dub.p, danc.p, want_table ? dpr.p : nullptr,
+                                want_table ? dal.p : nullptr, h->g.N, h->stream);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(h->stream);
+  if (e == cudaSuccess) e = cudaMemcpy(ancestors, danc.p, 4 * n, cudaMemcpyDeviceToHost);
+  if (e == cudaSuccess && want_table) e = cudaMemcpy(prob, dpr.p, 8 * n, cudaMemcpyDeviceToHost);
+  if (e == cudaSuccess && want_table) e = cudaMemcpy(alias, dal.p, 4 * n, cudaMemcpyDeviceToHost);
+  return sticky(h, e);
+}
+
+pf_status pf_debug_exchange(pf_handle* h, const float* logw, int64_t* src) {
+  if (!h || !logw || !src) return PF_EINVAL;
+  if (h->err != PF_OK) return h->err;
+  if (h->cfg.world != 1) return PF_ESTATE;
+  const long long M = h->g.M_local;
+  DevBuf<long long> dsrc;
+  cudaError_t e = dsrc.alloc(M);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(h->stream);
+  if (e == cudaSuccess) e = cudaMemcpy(h->logw, logw, sizeof(float) * M, cudaMemcpyHostToDevice);
+  if (e != cudaSuccess) return sticky(h, e);
+  const long long s = h->step > 0 ? h->step : 1;
+  pf_status st = publish(h, s);
+  if (st != PF_OK) return st;
+  pf::StepParams p = base_params(h, s + 1, pf::MODE_EXCHANGE);
+  p.dbg_src = dsrc.p;
+  st = launch(h, p);
+  if (st != PF_OK) return st;
+  h->step = s;
+  e = cudaStreamSynchronize(h->stream);
+  if (e == cudaSuccess) e = cudaMemcpy(src, dsrc.p, sizeof(long long) * M, cudaMemcpyDeviceToHost);
+  return sticky(h, e);
+}
+
+pf_status pf_set_trace(pf_handle* h, int32_t enable) {
+  if (!h) return PF_EINVAL;
+  if (enable && !h->trace) {
+    cudaError_t e = cudaStreamSynchronize(h->stream);
+    if (e == cudaSuccess) e = cudaMalloc(&h->d_src, sizeof(long long) * h->g.M_local);
+    if (e == cudaSuccess) e = cudaMalloc(&h->d_anc, sizeof(int) * h->g.M_local);
+    if (e != cudaSuccess) return sticky(h, e);
+    h->trace = true;
+  } else if (!enable && h->trace) {
+    cudaStreamSynchronize(h->stream);
+    cudaFree(h->d_src);
+    cudaFree(h->d_anc);
+    h->d_src = nullptr;
+    h->d_anc = nullptr;
+    h->trace = false;
+  }
+  return h->err;
+}
+
+pf_status pf_get_trace(pf_handle* h, int64_t* src, int32_t* ancestors) {
+  if (!h) return PF_EINVAL;
+  if (!h->trace) return PF_ESTATE;
+  cudaError_t e = cudaStreamSynchronize(h->stream);
+  if (e == cudaSuccess && src)
+    e = cudaMemcpy(src, h->d_src, sizeof(long long) * h->g.M_local, cudaMemcpyDeviceToHost);
+  if (e == cudaSuccess && ancestors)
+    e = cudaMemcpy(ancestors, h->d_anc, sizeof(int) * h->g.M_local, cudaMemcpyDeviceToHost);
+  return sticky(h, e);
+}
+
+pf_status pf_destroy(pf_handle* h) {
+  if (!h) return PF_OK;
+  if (h->stream || true) cudaStreamSynchronize(h->stream);
+  for (int i = 0; i < kStageSlots; ++i)
+    if (h->stage_ev[i]) cudaEventDestroy(h->stage_ev[i]);
+  if (h->pinned) cudaFreeHost(h->pinned);
+  if (h->d_src) cudaFree(h->d_src);
+  if (h->d_anc) cudaFree(h->d_anc);
+  delete h;
+  return PF_OK;
+}
+
+const char* pf_strerror(pf_status s) {
+  switch (s) {
+    case PF_OK: return "ok";
+    case PF_EINVAL: return "invalid argument or configuration";
+    case PF_ENOMEM: return "host allocation failed";
+    case PF_ECUDA: return "CUDA error";
+    case PF_ESTATE: return "call not valid in the handle's state";
+    case PF_EUNSUPPORTED: return "configuration not compiled (n_joints, m)";
+    default: return "unknown pf_status";
+  }
+}
+
+pf_status pf_last_error(const pf_handle* h) { return h ? h->err : PF_EINVAL; }
+
+int32_t pf_supported(int32_t* n_joints, int32_t* m, int32_t cap) {
+  const pf::KernelEntry* tables[] = {pf::kEntriesNJ2, pf::kEntriesNJ5, pf::kEntriesNJ28};
+  int32_t n = 0;
+  for (const pf::KernelEntry* t : tables)
+    for (int i = 0; i < pf::kNumEntriesPerNJ; ++i)
+      if (t[i].res == 0) {
+        if (n < cap && n_joints && m) {
+          n_joints[n] = t[i].nj;
+          m[n] = t[i].m;
+        }
+        ++n;
+      }
+  return n;
+}
+
+}  // extern "C"

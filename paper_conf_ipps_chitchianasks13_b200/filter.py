@@ -1,0 +1,173 @@
+"""ParticleFilter — torch-owned device buffers + the C-ABI handle.
+
+Torch is plumbing here: it allocates the caller-owned buffers of pf.h
+(pf_query_sizes) and provides the CUDA stream.  Every step of the hot path
+runs in libpf_b200.so; this class only marshals arguments (binding.py).
+"""
+from __future__ import annotations
+
+from dataclasses import dataclass
+
+import numpy as np
+import torch
+
+from . import binding as B
+
+TOPO = {"none": B.PF_TOPO_NONE, "ring": B.PF_TOPO_RING, "torus": B.PF_TOPO_TORUS2D}
+RESAMPLER = {"rws": B.PF_RESAMPLE_RWS, "vose": B.PF_RESAMPLE_VOSE}
+
+
+@dataclass
+class ArmModel:
+    """Robotic arm of PAPER.md:22–24 §VII-A, Table II defaults (readings R15, R16)."""
+    n_joints: int = 5
+    arm_length: float = 1.0
+    h_s: float = 0.1
+    sigma_theta: float = 0.1
+    sigma_pos: float = 0.1
+    sigma_vel: float = 0.1
+    sigma_cam: float = 0.1
+    sigma_theta_meas: float = 0.1
+
+    @property
+    def d(self) -> int:
+        return self.n_joints + 4
+
+    def c(self) -> B.pf_model_params:
+        return B.pf_model_params(B.PF_MODEL_ARM_PLANAR, self.n_joints, self.arm_length, self.h_s, self.sigma_theta,
+                                 self.sigma_pos, self.sigma_vel, self.sigma_cam, self.sigma_theta_meas)
+
+
+def _f32(a) -> np.ndarray:
+    return np.ascontiguousarray(a, dtype=np.float32)
+
+
+class ParticleFilter:
+    """Distributed particle filter (Algorithm 2) on one GPU shard.
+
+    Table I parameters: ``m`` particles per sub-filter,
+    ``n_filters`` (global N), exchange scheme ``topo`` and ``t`` particles per
+    exchange; ``resampler`` 'rws' | 'vose'.  ``rank``/``world`` select this
+    process's shard of the sub-filters (pf.h).
+    """
+
+    def __init__(self, mu0, sigma0, model: ArmModel | None = None, m: int = 256, n_filters: int = 4096,
+                 t: int = 1, topo: str = "ring", resampler: str = "rws", seed: int = 0, rank: int = 0,
+                 world: int = 1, torus_rows: int = 0, torus_cols: int = 0, device_inputs: bool = False,
+                 device: torch.device | int | None = None, stream: torch.cuda.Stream | None = None):
+        self.model = model or ArmModel()
+        self.device = torch.device("cuda", torch.cuda.current_device() if device is None else
+                                   (device if isinstance(device, int) else device.index or 0))
+        self.cfg = B.pf_config(m, n_filters, t, TOPO[topo], torus_rows, torus_cols, RESAMPLER[resampler],
+                               seed, rank, world, B.PF_DEVICE_INPUTS if device_inputs else 0)
+        self.m, self.n_filters, self.t, self.topo, self.resampler = m, n_filters, t, topo, resampler
+        self.rank, self.world = rank, world
+        self.d = self.model.d
+        self.nj = self.model.n_joints
+        mc = self.model.c()
+        sizes = B.pf_query_sizes(self.cfg, mc)
+        with torch.cuda.device(self.device):
+            self.stream = stream or torch.cuda.current_stream(self.device)
+            alloc = lambda n: torch.empty(max(int(n), 16), dtype=torch.uint8, device=self.device)
+            self._state = alloc(sizes.state)
+            self._logw = alloc(sizes.logw)
+            self._mailbox = alloc(sizes.mailbox)
+            self._scratch = alloc(sizes.scratch)
+            bufs = B.pf_buffers(self._state.data_ptr(), self._logw.data_ptr(), self._mailbox.data_ptr(),
+                                self._scratch.data_ptr())
+            self.h = B.pf_init(self.cfg, mc, bufs, self.stream.cuda_stream, _f32(mu0), _f32(sigma0))
+        self.shard = B.pf_get_shard(self.h)
+        self.M_local = self.shard.n_local * m
+        self._xhat = np.zeros(self.d, np.float32)
+
+    # -- views of the caller-owned buffers (torch, device) -------------------
+    @property
+    def state(self) -> torch.Tensor:
+        return self._state[: 4 * self.d * self.M_local].view(torch.float32).view(self.d, self.M_local)
+
+    @property
+    def logw(self) -> torch.Tensor:
+        return self._logw[: 4 * self.M_local].view(torch.float32)
+
+    @property
+    def mailbox(self) -> torch.Tensor:
+        s = self.shard
+        n = 2 * s.n_ext * s.t * s.entry_floats
+        return self._mailbox[: 4 * n].view(torch.float32).view(2, s.n_ext, s.t, s.entry_floats)
+
+    @property
+    def record(self) -> torch.Tensor:
+        ptr, n = B.pf_record_ptr(self.h)
+        off = ptr - self._scratch.data_ptr()
+        return self._scratch[off: off + 4 * n].view(torch.float32)
+
+    # -- the path -----------------------------------------------------------
+    def step(self, z, u) -> None:
+        """One time step (host numpy z/u, or device tensors with device_inputs)."""
+        if self.cfg.flags & B.PF_DEVICE_INPUTS:
+            B.pf_step(self.h, z.data_ptr(), u.data_ptr())
+        else:
+            B.pf_step(self.h, _f32(z), _f32(u))
+
+    def step_batch(self, zs: torch.Tensor, us: torch.Tensor, est: torch.Tensor | None = None) -> None:
+        """T steps with device-resident inputs zs [T][nj+2], us [T][nj]; est [T][4+d]."""
+        assert zs.is_cuda and us.is_cuda and zs.dtype == torch.float32 and us.dtype == torch.float32
+        B.pf_step_batch(self.h, zs.shape[0], zs.data_ptr(), us.data_ptr(), None if est is None else est.data_ptr())
+
+    def estimate(self):
+        """(x_hat [d], logw, global index) of the particle with the highest weight."""
+        lw, idx = B.pf_estimate(self.h, self._xhat)
+        return self._xhat.copy(), lw, idx
+
+    def reduce_records(self, records: torch.Tensor) -> None:
+        B.pf_reduce_records(self.h, records.data_ptr(), records.shape[0])
+
+    def get_particles(self):
+        s = np.zeros((self.d, self.M_local), np.float32)
+        w = np.zeros(self.M_local, np.float32)
+        k = B.pf_get_particles(self.h, s, w)
+        return s, w, k
+
+    def set_particles(self, state, logw, step: int) -> None:
+        B.pf_set_particles(self.h, _f32(state), _f32(logw), step)
+
+    # -- test hooks ----------------------------------------------------------
+    def debug_sample_weight(self, state_in, z, u, k: int):
+        s_out = np.zeros((self.d, self.M_local), np.float32)
+        w_out = np.zeros(self.M_local, np.float32)
+        B.pf_debug_sample_weight(self.h, _f32(state_in), _f32(z), _f32(u), k, s_out, w_out)
+        return s_out, w_out
+
+    def debug_resample(self, q, ua, ub):
+        q = np.ascontiguousarray(q, np.uint32)
+        anc = np.zeros(q.shape, np.int32)
+        prob = np.zeros(q.shape, np.uint64)
+        alias = np.zeros(q.shape, np.int32)
+        B.pf_debug_resample(self.h, q, np.ascontiguousarray(ua, np.uint32), np.ascontiguousarray(ub, np.uint32),
+                            anc, prob, alias)
+        return anc, prob, alias
+
+    def debug_exchange(self, logw):
+        src = np.zeros(self.M_local, np.int64)
+        B.pf_debug_exchange(self.h, _f32(logw), src)
+        return src
+
+    def set_trace(self, enable: bool = True) -> None:
+        B.pf_set_trace(self.h, enable)
+
+    def trace(self):
+        src = np.zeros(self.M_local, np.int64)
+        anc = np.zeros(self.M_local, np.int32)
+        B.pf_get_trace(self.h, src, anc)
+        return src, anc
+
+    def close(self) -> None:
+        if getattr(self, "h", None):
+            B.pf_destroy(self.h)
+            self.h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass

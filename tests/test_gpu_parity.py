@@ -1,0 +1,187 @@
+"""CUDA path (libpf_b200.so through the C ABI) vs the CPU oracle, element by
+element on the same seeded inputs.  Bar (north_star, R18): indices and
+exchange permutations bit-exact; states / log-weights / estimates within
+1e-5 relative — and, because both sides follow the fp32 contract F1–F11,
+the whole trajectory is expected to be bit-identical (asserted separately)."""
+import numpy as np
+import pytest
+
+pytestmark = pytest.mark.gpu
+
+TOL = 1e-5
+
+
+def _close(a, b):
+    a, b = np.asarray(a, np.float64), np.asarray(b, np.float64)
+    assert np.all(np.abs(a - b) <= TOL * np.maximum(1.0, np.abs(b))), float(np.max(np.abs(a - b)))
+
+
+@pytest.fixture(scope="module")
+def P():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    from paper_conf_ipps_chitchianasks13_b200 import build, filter as F
+    build.build()
+    return F
+
+
+def _pair(P, orc, W, nj, m, N, t=1, topo="ring", res="rws", seed=1, T=100, traj_seed=0):
+    tr = W.make_trajectory(nj, T, traj_seed)
+    g = P.ParticleFilter(tr["mu0"], tr["sigma0"], P.ArmModel(n_joints=nj), m=m, n_filters=N, t=t, topo=topo,
+                         resampler=res, seed=seed)
+    o = orc.Filter(orc.Config(m=m, n_filters=N, t=t, topo=topo, resampler=res, seed=seed),
+                   orc.Model(n_joints=nj), tr["mu0"], tr["sigma0"])
+    return tr, g, o
+
+
+def test_init_prior_bit_exact(P, orc, W):
+    tr, g, o = _pair(P, orc, W, 5, 64, 8, seed=(5 << 32) | 3)
+    sg, _, kg = g.get_particles()
+    so, _, ko = o.get()
+    assert kg == ko == 0
+    np.testing.assert_array_equal(sg, so)
+
+
+@pytest.mark.parametrize("nj,m,N", [(2, 64, 16), (5, 256, 4), (28, 32, 8), (5, 1024, 2), (28, 256, 2)])
+def test_sample_weight(P, orc, W, nj, m, N):
+    tr = W.make_trajectory(nj, 10, 1)
+    g = P.ParticleFilter(tr["mu0"], tr["sigma0"], P.ArmModel(n_joints=nj), m=m, n_filters=N, seed=77)
+    s_in = W.random_particles(tr, m * N, nj)
+    for k in (1, 7):
+        sg, wg = g.debug_sample_weight(s_in, tr["Z"][k], tr["U"][k - 1], k)
+        so, wo = orc.sample_weight(orc.Model(n_joints=nj), 77, s_in, tr["Z"][k], tr["U"][k - 1], k)
+        _close(sg, so)
+        _close(wg, wo)
+        np.testing.assert_array_equal(sg, so)     # fp32 contract: bit-identical
+        np.testing.assert_array_equal(wg, wo)
+
+
+@pytest.mark.parametrize("res", ["rws", "vose"])
+@pytest.mark.parametrize("m", [32, 64, 256, 1024])
+@pytest.mark.parametrize("kind", ["mixed", "uniform", "onehot"])
+def test_resample_bit_exact(P, orc, W, res, m, kind):
+    N = 24
+    tr = W.make_trajectory(2, 4, 0)
+    g = P.ParticleFilter(tr["mu0"], tr["sigma0"], P.ArmModel(n_joints=2), m=m, n_filters=N, resampler=res)
+    q = W.random_q(N, m, m + len(kind), kind)
+    if kind == "mixed":
+        q[::3, ::2] = 0          # zero-weight slots (never drawn)
+    rng = np.random.default_rng(m)
+    ua = rng.integers(0, 2**32, (N, m), dtype=np.uint64).astype(np.uint32)
+    ub = rng.integers(0, 2**32, (N, m), dtype=np.uint64).astype(np.uint32)
+    ua[0, :4] = [0, 0xFFFFFFFF, 0x80000000, 1]
+    anc, prob, alias = g.debug_resample(q, ua, ub)
+    np.testing.assert_array_equal(anc, orc.resample_q(q, res, ua, ub))
+    if res == "vose":
+        for n in range(N):
+            p_o, a_o = orc.vose_build(q[n])
+            np.testing.assert_array_equal(prob[n], p_o)
+            np.testing.assert_array_equal(alias[n], a_o)
+
+
+@pytest.mark.parametrize("topo,N,m,t", [("ring", 16, 64, 1), ("ring", 8, 32, 3), ("torus", 16, 64, 2),
+                                         ("torus", 8, 128, 1), ("ring", 2, 32, 1), ("torus", 4, 32, 1),
+                                         ("ring", 1, 32, 2)])
+def test_exchange_bit_exact(P, orc, W, topo, N, m, t):
+    tr = W.make_trajectory(2, 4, 0)
+    g = P.ParticleFilter(tr["mu0"], tr["sigma0"], P.ArmModel(n_joints=2), m=m, n_filters=N, t=t, topo=topo)
+    for s in range(3):
+        w = W.random_logw(N, m, 100 + s, ties=(s != 1))
+        src = g.debug_exchange(w.ravel())
+        np.testing.assert_array_equal(src.reshape(N, m),
+                                      orc.exchange(orc.Config(m=m, n_filters=N, t=t, topo=topo), w))
+
+
+def _run_compare(P, orc, W, nj, m, N, T, **kw):
+    tr, g, o = _pair(P, orc, W, nj, m, N, T=T, **kw)
+    g.set_trace(True)
+    for k in range(1, T + 1):
+        g.step(tr["Z"][k], tr["U"][k - 1])
+        o.step(tr["Z"][k], tr["U"][k - 1])
+        xg, lg, ig = g.estimate()
+        xo, lo, io = o.estimate()
+        assert ig == io, f"estimate index differs at step {k}"
+        _close(xg, xo)
+        _close(lg, lo)
+        if k in (1, 2, T):
+            src_g, anc_g = g.trace()
+            src_o, anc_o = o.trace()
+            np.testing.assert_array_equal(src_g, src_o)
+            np.testing.assert_array_equal(anc_g, anc_o)
+            sg, wg, kg = g.get_particles()
+            so, wo, ko = o.get()
+            assert kg == ko == k
+            _close(sg, so)
+            _close(wg, wo)
+            np.testing.assert_array_equal(sg, so)
+            np.testing.assert_array_equal(wg, wo)
+    return g, o
+
+
+def test_full_filter_c1(P, orc, W):
+    # BASELINE config 1: 2-link arm, 16 sub-filters x 64, RWS, ring t = 1, 100 steps
+    _run_compare(P, orc, W, 2, 64, 16, 100)
+
+
+@pytest.mark.parametrize("nj,m,N,t,topo,res", [
+    (2, 64, 16, 1, "torus", "vose"),
+    (5, 256, 16, 2, "ring", "vose"),
+    (5, 128, 64, 1, "torus", "rws"),
+    (5, 32, 32, 0, "none", "rws"),
+    (28, 64, 8, 1, "ring", "vose"),
+    (5, 1024, 4, 4, "torus", "rws"),
+])
+def test_full_filter_variants(P, orc, W, nj, m, N, t, topo, res):
+    _run_compare(P, orc, W, nj, m, N, 12, t=t, topo=topo, res=res, seed=nj * 1000 + m)
+
+
+def test_set_particles_resume(P, orc, W):
+    # checkpoint / resume from a generator-made weighted set, then 5 steps
+    nj, m, N = 5, 64, 16
+    tr, g, o = _pair(P, orc, W, nj, m, N, T=20, res="vose", topo="torus")
+    s0 = W.random_particles(tr, m * N, 9)
+    w0 = W.random_logw(N, m, 9).ravel()
+    g.set_particles(s0, w0, 7)
+    o.set(s0, w0, 7)
+    for k in range(8, 13):
+        g.step(tr["Z"][k], tr["U"][k - 1])
+        o.step(tr["Z"][k], tr["U"][k - 1])
+        assert g.estimate()[2] == o.estimate()[2]
+    np.testing.assert_array_equal(g.get_particles()[0], o.get()[0])
+
+
+@pytest.mark.parametrize("res", ["rws", "vose"])
+def test_full_size_c2(P, orc, W, res):
+    # BASELINE config 2 at full size: medium arm, 4096 x 256 = 2^20, ring t=1,
+    # in the launch configuration bench.py times; 3 steps vs the oracle
+    tr, g, o = _pair(P, orc, W, 5, 256, 4096, T=10, res=res, seed=2013)
+    for k in range(1, 4):
+        g.step(tr["Z"][k], tr["U"][k - 1])
+        o.step(tr["Z"][k], tr["U"][k - 1])
+        xg, lg, ig = g.estimate()
+        xo, lo, io = o.estimate()
+        assert ig == io
+        np.testing.assert_array_equal(xg, xo)
+    sg, wg, _ = g.get_particles()
+    so, wo, _ = o.get()
+    np.testing.assert_array_equal(sg, so)
+    np.testing.assert_array_equal(wg, wo)
+
+
+def test_step_batch_matches_streaming(P, W):
+    import torch
+    nj, m, N, T = 5, 128, 32, 20
+    tr = W.make_trajectory(nj, T, 3)
+    a = P.ParticleFilter(tr["mu0"], tr["sigma0"], P.ArmModel(n_joints=nj), m=m, n_filters=N, seed=9)
+    b = P.ParticleFilter(tr["mu0"], tr["sigma0"], P.ArmModel(n_joints=nj), m=m, n_filters=N, seed=9)
+    zs = torch.tensor(tr["Z"][1:T + 1], device="cuda")
+    us = torch.tensor(tr["U"][0:T], device="cuda")
+    est = torch.zeros(T, 4 + nj + 4, device="cuda")
+    b.step_batch(zs, us, est)
+    torch.cuda.synchronize()
+    for k in range(1, T + 1):
+        a.step(tr["Z"][k], tr["U"][k - 1])
+        x, lw, idx = a.estimate()
+        np.testing.assert_array_equal(est[k - 1, 4:].cpu().numpy(), x)
+        assert est[k - 1, 2].item() == lw
