@@ -403,8 +403,8 @@ __global__ void __launch_bounds__(M) pf_step_kernel(const __grid_constant__ Step
         P.dbg_src[n * M + tid] = src;
       }
       __syncthreads();
-    } else if (do_merge && P.dbg_src) {
-      P.dbg_src[n * M + tid] = pidx;
+    } else if ((do_merge || mode == MODE_STEP) && P.dbg_src) {
+      P.dbg_src[n * M + tid] = pidx;   // no exchange (k = 1 or deg*t = 0): identity
     }
 
     if (mode == MODE_EXCHANGE) {
