@@ -19,11 +19,14 @@
  *    handle's stream; only pf_estimate / pf_get_particles / the debug hooks
  *    synchronize it.
  *  - A handle is used by one host thread at a time.
- *  - Layouts: particle state is SoA, float32 [d][M_local] (row c holds state
- *    component c of every local particle; d = n_joints + 4, components
- *    theta_0..theta_{n_j-1}, x, y, v_x, v_y — PAPER.md:22 §VII-A); local
- *    particle column = n_local * m + i for sub-filter n_local, slot i; the
- *    log-weight ("logw", reading R7) is float32 [M_local].
+ *  - Device layout (blocked SoA): the particle buffer is float32
+ *    [n_local][d+1][m] — for every local sub-filter one contiguous block
+ *    whose rows 0..d-1 are the state components (d = n_joints + 4:
+ *    theta_0..theta_{n_j-1}, x, y, v_x, v_y — PAPER.md:22 §VII-A) of its m
+ *    particles and whose row d is their log-weight (reading R7).
+ *  - Host layout (get/set/debug hooks): state float32 [d][M_local] (row c =
+ *    component c of every local particle, column n_local*m + i for
+ *    sub-filter n_local, slot i), log-weights float32 [M_local].
  */
 #ifndef PF_H
 #define PF_H
@@ -88,15 +91,13 @@ typedef struct {
 
 /* Bytes of each caller-owned device buffer. */
 typedef struct {
-  uint64_t state;    /* float [d][M_local]                                          */
-  uint64_t logw;     /* float [M_local]                                             */
+  uint64_t state;    /* float [n_local][d+1][m]: states + log-weights (blocked SoA) */
   uint64_t mailbox;  /* float [2][n_ext][max(t,1)][d+2]: exchange mailbox, see below */
   uint64_t scratch;  /* keys, counters, estimate record, step inputs                */
 } pf_sizes;
 
 typedef struct {
   void* state;
-  void* logw;
   void* mailbox;
   void* scratch;
 } pf_buffers;
@@ -174,9 +175,9 @@ pf_status pf_reduce_records(pf_handle* h, const float* records_dev, int32_t coun
 /* Shard geometry and mailbox layout for halo exchange. */
 pf_status pf_get_shard(const pf_handle* h, pf_shard* out);
 
-/* Checkpoint: copy the weighted particle set of the last step (state
- * [d][M_local], logw [M_local], host) and its step index (step 0 = prior,
- * logw undefined).  Synchronizes. */
+/* Checkpoint: copy the weighted particle set of the last step (host layout:
+ * state [d][M_local], logw [M_local]) and its step index (step 0 = prior,
+ * logw = 0).  Synchronizes. */
 pf_status pf_get_particles(pf_handle* h, float* state_host, float* logw_host, int64_t* step);
 /* Resume: load a weighted particle set as the result of step `step` >= 1
  * (host pointers), republish its best t to the mailbox and its estimate.

@@ -40,11 +40,11 @@ class pf_config(C.Structure):
 
 
 class pf_sizes(C.Structure):
-    _fields_ = [("state", C.c_uint64), ("logw", C.c_uint64), ("mailbox", C.c_uint64), ("scratch", C.c_uint64)]
+    _fields_ = [("state", C.c_uint64), ("mailbox", C.c_uint64), ("scratch", C.c_uint64)]
 
 
 class pf_buffers(C.Structure):
-    _fields_ = [("state", C.c_void_p), ("logw", C.c_void_p), ("mailbox", C.c_void_p), ("scratch", C.c_void_p)]
+    _fields_ = [("state", C.c_void_p), ("mailbox", C.c_void_p), ("scratch", C.c_void_p)]
 
 
 class pf_shard(C.Structure):

@@ -1,8 +1,8 @@
-// pf_inst_nj2.cu — pf_step_kernel instantiations for the n_joints = 2 arm
-// (d = 6), every m in {32..1024}, RWS and Vose.
+// pf_inst_nj2.cu — pf_step_kernel instantiations for the 2-link arm (d = 6).
 #include "pf_kernels.cuh"
 #include "pf_registry.h"
 
 namespace pf {
-const KernelEntry kEntriesNJ2[] = {PF_ENTRIES_FOR(2)};
+const KernelEntry kEntriesNJ2[] = {PF_SMALL_D_ENTRIES(2, 0), PF_SMALL_D_ENTRIES(2, 1)};
+const int kNumEntriesNJ2 = sizeof(kEntriesNJ2) / sizeof(kEntriesNJ2[0]);
 }  // namespace pf

@@ -1,8 +1,18 @@
-// pf_inst_nj28.cu — pf_step_kernel instantiations for the n_joints = 28 arm
-// (d = 32), every m in {32..1024}, RWS and Vose.
+// pf_inst_nj28.cu — pf_step_kernel instantiations for the high-DOF arm
+// (28 joints, d = 32; config C4): larger groups (fewer particles per thread)
+// because a sub-filter's state block is 4 (d+1) m bytes of shared memory.
 #include "pf_kernels.cuh"
 #include "pf_registry.h"
 
 namespace pf {
-const KernelEntry kEntriesNJ28[] = {PF_ENTRIES_FOR(28)};
+#define PF_LARGE_D_ENTRIES(NJ, RES)                                                                       \
+  PF_ENTRY(NJ, 32, RES, 1, 4, 1, 1), PF_ENTRY(NJ, 64, RES, 2, 2, 1, 1), PF_ENTRY(NJ, 128, RES, 4, 1, 1, 1), \
+      PF_ENTRY(NJ, 256, RES, 8, 1, 1, 1), PF_ENTRY(NJ, 512, RES, 16, 1, 1, 1),                             \
+      PF_ENTRY(NJ, 1024, RES, 16, 1, 1, 1)
+const KernelEntry kEntriesNJ28[] = {
+    PF_LARGE_D_ENTRIES(28, 0), PF_LARGE_D_ENTRIES(28, 1),
+    PF_ENTRY(28, 256, 0, 4, 1, 1, 1), PF_ENTRY(28, 256, 0, 8, 1, 2, 1), PF_ENTRY(28, 256, 0, 2, 2, 1, 1),
+    PF_ENTRY(28, 256, 1, 4, 1, 1, 1), PF_ENTRY(28, 256, 1, 8, 1, 2, 1),
+};
+const int kNumEntriesNJ28 = sizeof(kEntriesNJ28) / sizeof(kEntriesNJ28[0]);
 }  // namespace pf

@@ -1,8 +1,14 @@
-// pf_inst_nj5.cu — pf_step_kernel instantiations for the n_joints = 5 arm
-// (d = 9), every m in {32..1024}, RWS and Vose.
+// pf_inst_nj5.cu — pf_step_kernel instantiations for the paper's medium arm
+// (5 joints incl. the base, d = 9; Table II), with alternative
+// mappings of m = 256 (configs C2 / C5) for tuning.
 #include "pf_kernels.cuh"
 #include "pf_registry.h"
 
 namespace pf {
-const KernelEntry kEntriesNJ5[] = {PF_ENTRIES_FOR(5)};
+const KernelEntry kEntriesNJ5[] = {
+    PF_SMALL_D_ENTRIES(5, 0), PF_SMALL_D_ENTRIES(5, 1),
+    PF_ENTRY(5, 256, 0, 8, 1, 2, 1), PF_ENTRY(5, 256, 0, 2, 4, 1, 1), PF_ENTRY(5, 256, 0, 1, 8, 1, 1),
+    PF_ENTRY(5, 256, 0, 4, 2, 2, 2), PF_ENTRY(5, 256, 1, 8, 1, 2, 1), PF_ENTRY(5, 256, 1, 2, 4, 1, 1),
+};
+const int kNumEntriesNJ5 = sizeof(kEntriesNJ5) / sizeof(kEntriesNJ5[0]);
 }  // namespace pf

@@ -1,7 +1,7 @@
 // pf_kernels.cuh — sm_100a kernels of the distributed particle filter.
 //
-// pf_step_kernel<NJ, M, RES> is the ROTATED STEP: launch k
-// performs, for every sub-filter of this shard,
+// pf_step_kernel<Cfg> is the ROTATED STEP: launch k performs,
+// for every sub-filter of this shard,
 //   a6 exchange   merge the neighbours' best t of step k-1 (mailbox) into the
 //                 own worst deg*t slots                  (Alg.2 l.10–14, R2–R5)
 //   a7 normalise  q_i = floor(2^22 exp(l_i - l_max))     (§VI-F, R7–R8)
@@ -15,16 +15,22 @@
 //   a10 store state + log-weight (in place)
 // so each launch streams the particle set through HBM once (read + write).
 //
-// Mapping: one CTA of M threads per sub-filter (one thread per particle, as
-// the paper's one work-group per sub-filter, §VI), persistent
-// grid-stride loop over the shard's sub-filters.  A sub-filter's d state
-// rows and log-weight row (SoA, contiguous m floats each) are brought into
-// shared memory by d+1 TMA bulk copies (cp.async.bulk + mbarrier); all
-// reductions / scans are warp-shuffle / REDUX + one cross-warp level.
+// Data layout (blocked SoA): sub-filter n of the shard owns one contiguous
+// block of (D+1) rows x M floats — rows 0..D-1 the state components, row D
+// the log-weight — so a sub-filter arrives in shared memory with ONE TMA bulk
+// copy and every per-component store is a coalesced row store at an
+// immediate offset.
+//
+// Mapping: a GROUP of GW warps owns one sub-filter at a time (GW = 1: one
+// warp per sub-filter, no CTA barrier at all); thread t of the group owns the
+// P = M / (32 GW) strided slots t, t + 32GW, ...; a CTA holds S groups;
+// persistent grid-stride loop over sub-filters; NSTAGE = 2 double-buffers the
+// TMA load of the group's next sub-filter behind the current one.
 #pragma once
 #include <cuda_runtime.h>
 
 #include <cstdint>
+#include <type_traits>
 
 #include "pf_device.cuh"
 
@@ -38,9 +44,7 @@ enum : int { RES_RWS = 0, RES_VOSE = 1 };
 
 struct StepParams {
   ArmConsts mc;
-  float* state;            // [d][stride]
-  float* logw;             // [stride]
-  long long stride;        // M_local
+  float* parts;            // [n_local][D+1][M] blocked SoA (row D = log-weight)
   const float* mb_prev;    // mailbox parity (k-1)&1 : [n_ext][tt][E]
   float* mb_cur;           // mailbox parity k&1
   const float* z;          // [NJ+2] device
@@ -54,8 +58,9 @@ struct StepParams {
   int* dbg_anc;            // nullable [M_local] ancestors
   long long n_local, g0, n_global, R, C;
   int t, tt, topo, deg;
-  uint32_t key0, key1, k;
+  uint32_t k;
   int mode, first;
+  uint32_t rk[20];         // Philox round keys (key0 + r W0, key1 + r W1), r = 0..9
 };
 
 // ------------------------------------------------------------- PTX helpers
@@ -92,86 +97,152 @@ __device__ __forceinline__ void mbar_wait(u64* bar, uint32_t parity) {
       : "memory");
 }
 
-// ------------------------------------------------------ block primitives
-// All take the two-slot reduction buffer `red` ([2][32] u64) and a uniform
-// buffer toggle; every call with NW > 1 contains one __syncthreads, which
-// makes a slot reusable two calls later.
-template <int NW>
-__device__ __forceinline__ u64 block_max_u64(u64 v, u64* red, int& rb) {
-  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  uint32_t hi = __reduce_max_sync(0xFFFFFFFFu, static_cast<uint32_t>(v >> 32));
-  uint32_t lo = __reduce_max_sync(0xFFFFFFFFu, (static_cast<uint32_t>(v >> 32) == hi) ? static_cast<uint32_t>(v) : 0u);
-  if (NW == 1) return (static_cast<u64>(hi) << 32) | lo;
-  u64* r = red + rb * 32;
-  rb ^= 1;
-  if (lane == 0) r[warp] = (static_cast<u64>(hi) << 32) | lo;
-  __syncthreads();
-  const u64 w = lane < NW ? r[lane] : 0ull;
-  hi = __reduce_max_sync(0xFFFFFFFFu, static_cast<uint32_t>(w >> 32));
-  lo = __reduce_max_sync(0xFFFFFFFFu, (static_cast<uint32_t>(w >> 32) == hi) ? static_cast<uint32_t>(w) : 0u);
+// ------------------------------------------------------- configuration
+// NJ joints (D = NJ + 4), M particles per sub-filter, resampler RES; a group
+// of GW warps owns one sub-filter; S groups per CTA; NSTAGE TMA stages per
+// group; the per-particle sample/weight loop over a thread's P slots is
+// unrolled UNR times (P for full unrolling; 1 keeps one copy of the
+// ~10–40 KB per-particle code in the instruction cache).
+template <int NJ_, int M_, int RES_, int GW_, int S_, int NSTAGE_, int UNR_>
+struct KCfg {
+  static constexpr int NJ = NJ_, M = M_, RES = RES_, GW = GW_, S = S_, NSTAGE = NSTAGE_, UNR = UNR_;
+  static constexpr int D = NJ + 4;
+  static constexpr int E = D + 2;            // mailbox entry: [logw, index bits, x_0..x_{D-1}]
+  static constexpr int T = 32 * GW;          // threads per group
+  static constexpr int P = M / T;            // particles per thread
+  static constexpr int ROW = (D + 1) * M;    // floats per sub-filter block
+  static constexpr bool SCAN32 = (M <= 512);  // Q <= M 2^22 fits 32 bits
+  static constexpr bool STAGED = UNR < P;    // rolled sample loop: per-slot values via smem
+  static_assert(P >= 1 && P * T == M, "M must be a multiple of the group size");
+  static_assert(P <= 32, "exclusion masks are 32-bit");
+  static_assert(S >= 1 && S <= 15, "named barriers 1..S");
+  static constexpr int KMAX = 32;            // deg * t <= 32 (validated by the runtime)
+  // per-group shared memory
+  static constexpr size_t stage_bytes = sizeof(float) * ROW;
+  static constexpr size_t g_stage = 0;
+  static constexpr size_t g_scan = NSTAGE * stage_bytes;                          // u64 [M]
+  static constexpr size_t g_slot = g_scan + sizeof(u64) * M;                      // int anc[M], u32 bz[M], bw[M]
+  static constexpr size_t g_prob = g_slot + (STAGED ? 12 * M : 0);                // u64 [M]  (Vose)
+  static constexpr size_t g_alias = g_prob + (RES == RES_VOSE ? sizeof(u64) * M : 0);
+  static constexpr size_t g_lists = g_alias + (RES == RES_VOSE ? sizeof(int) * M : 0);
+  static constexpr size_t g_red = g_lists + (RES == RES_VOSE ? sizeof(int) * M : 0);   // u64 [2][64]
+  static constexpr size_t g_cand = g_red + sizeof(u64) * 128;                    // u64 [GW][KMAX+1]
+  static constexpr size_t g_misc = g_cand + sizeof(u64) * GW * (KMAX + 1);       // int [GW][KMAX]
+  static constexpr size_t g_bar = g_misc + sizeof(int) * GW * KMAX;              // u64 [2]
+  static constexpr size_t group_bytes = (g_bar + 16 + 127) / 128 * 128;
+  // per-CTA
+  static constexpr size_t c_zin = 0;          // float [64]: z (NJ+2), h_s u (NJ)
+  static constexpr size_t c_groups = 256;
+  static constexpr size_t smem = c_groups + S * group_bytes;
+  // slot j of group thread t: strided, so chunk j of the group covers the
+  // contiguous slots [jT, (j+1)T) and every row store is coalesced
+  __device__ __forceinline__ static int slot(int t, int j) { return j * T + t; }
+};
+
+// ------------------------------------------------------- group primitives
+template <int GW>
+__device__ __forceinline__ void gsync(int g) {
+  if constexpr (GW == 1) {
+    __syncwarp();
+  } else {
+    asm volatile("bar.sync %0, %1;" ::"r"(g + 1), "n"(32 * GW) : "memory");
+  }
+}
+
+struct GroupCtx {
+  int g;          // group index in the CTA
+  int t;          // thread index in the group
+  int lane, wig;  // lane, warp in group
+  u64* red;       // [2][64] cross-warp reduction slots
+  int rb;         // slot toggle (uniform in the group); each call with GW > 1
+                  // syncs once, so a slot is reusable two calls later
+};
+
+__device__ __forceinline__ u64 warp_max_u64(u64 v) {
+  const uint32_t hi = __reduce_max_sync(0xFFFFFFFFu, static_cast<uint32_t>(v >> 32));
+  const uint32_t lo =
+      __reduce_max_sync(0xFFFFFFFFu, (static_cast<uint32_t>(v >> 32) == hi) ? static_cast<uint32_t>(v) : 0u);
+  return (static_cast<u64>(hi) << 32) | lo;
+}
+__device__ __forceinline__ u64 warp_min_u64(u64 v) {
+  const uint32_t hi = __reduce_min_sync(0xFFFFFFFFu, static_cast<uint32_t>(v >> 32));
+  const uint32_t lo = __reduce_min_sync(
+      0xFFFFFFFFu, (static_cast<uint32_t>(v >> 32) == hi) ? static_cast<uint32_t>(v) : 0xFFFFFFFFu);
   return (static_cast<u64>(hi) << 32) | lo;
 }
 
-template <int NW>
-__device__ __forceinline__ u64 block_min_u64(u64 v, u64* red, int& rb) {
-  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  uint32_t hi = __reduce_min_sync(0xFFFFFFFFu, static_cast<uint32_t>(v >> 32));
-  uint32_t lo = __reduce_min_sync(0xFFFFFFFFu,
-                                  (static_cast<uint32_t>(v >> 32) == hi) ? static_cast<uint32_t>(v) : 0xFFFFFFFFu);
-  if (NW == 1) return (static_cast<u64>(hi) << 32) | lo;
-  u64* r = red + rb * 32;
-  rb ^= 1;
-  if (lane == 0) r[warp] = (static_cast<u64>(hi) << 32) | lo;
-  __syncthreads();
-  const u64 w = lane < NW ? r[lane] : ~0ull;
-  hi = __reduce_min_sync(0xFFFFFFFFu, static_cast<uint32_t>(w >> 32));
-  lo = __reduce_min_sync(0xFFFFFFFFu,
-                         (static_cast<uint32_t>(w >> 32) == hi) ? static_cast<uint32_t>(w) : 0xFFFFFFFFu);
-  return (static_cast<u64>(hi) << 32) | lo;
+template <int GW>
+__device__ __forceinline__ u64 gmax_u64(u64 v, GroupCtx& G) {
+  const u64 w = warp_max_u64(v);
+  if constexpr (GW == 1) {
+    return w;
+  } else {
+    u64* r = G.red + G.rb * 64;
+    G.rb ^= 1;
+    if (G.lane == 0) r[G.wig] = w;
+    gsync<GW>(G.g);
+    return warp_max_u64(G.lane < GW ? r[G.lane] : 0ull);
+  }
 }
 
-template <int NW>
-__device__ __forceinline__ uint32_t block_max_u32(uint32_t v, u64* red, int& rb) {
-  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  uint32_t m = __reduce_max_sync(0xFFFFFFFFu, v);
-  if (NW == 1) return m;
-  u64* r = red + rb * 32;
-  rb ^= 1;
-  if (lane == 0) r[warp] = m;
-  __syncthreads();
-  return __reduce_max_sync(0xFFFFFFFFu, lane < NW ? static_cast<uint32_t>(r[lane]) : 0u);
-}
-
-__device__ __forceinline__ u64 warp_incl_scan_u64(u64 x) {
-  const int lane = threadIdx.x & 31;
+template <typename X>
+__device__ __forceinline__ X warp_incl_scan(X x, int lane) {
 #pragma unroll
   for (int o = 1; o < 32; o <<= 1) {
-    const u64 y = __shfl_up_sync(0xFFFFFFFFu, x, o);
+    const X y = __shfl_up_sync(0xFFFFFFFFu, x, o);
     if (lane >= o) x += y;
   }
   return x;
 }
 
-// Exclusive prefix sum over threads in tid order; `total` = block sum.
-template <int NW>
-__device__ __forceinline__ u64 block_excl_scan_u64(u64 v, u64* red, int& rb, u64& total) {
-  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  const u64 x = warp_incl_scan_u64(v);
-  if (NW == 1) {
-    total = __shfl_sync(0xFFFFFFFFu, x, 31);
-    return x - v;
+// Slot-order inclusive prefix of per-slot values val[P] over the group
+// (strided slots, KCfg::slot): out[j] = sum of val over slots <= slot(t, j).
+// Returns the group total.  One group barrier when GW > 1.
+template <class C, typename X>
+__device__ __forceinline__ X slot_scan_incl(const X (&val)[C::P], X (&out)[C::P], GroupCtx& G) {
+  constexpr int P = C::P, GW = C::GW;
+  X w[P];
+#pragma unroll
+  for (int j = 0; j < P; ++j) w[j] = val[j];
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+#pragma unroll
+    for (int j = 0; j < P; ++j) {
+      const X y = __shfl_up_sync(0xFFFFFFFFu, w[j], o);
+      if (G.lane >= o) w[j] += y;
+    }
   }
-  u64* r = red + rb * 32;
-  rb ^= 1;
-  if (lane == 31) r[warp] = x;
-  __syncthreads();
-  const u64 wt = warp_incl_scan_u64(lane < NW ? r[lane] : 0ull);
-  const u64 off = __shfl_sync(0xFFFFFFFFu, wt, (warp + 31) & 31);
-  total = __shfl_sync(0xFFFFFFFFu, wt, NW - 1);
-  return (warp > 0 ? off : 0ull) + x - v;
+  if constexpr (GW == 1) {
+    X base = 0;
+#pragma unroll
+    for (int j = 0; j < P; ++j) {
+      out[j] = base + w[j];
+      base += __shfl_sync(0xFFFFFFFFu, w[j], 31);
+    }
+    return base;
+  } else {
+    X* r = reinterpret_cast<X*>(G.red + G.rb * 64);
+    G.rb ^= 1;
+    if (G.lane == 31) {
+#pragma unroll
+      for (int j = 0; j < P; ++j) r[j * GW + G.wig] = w[j];
+    }
+    gsync<GW>(G.g);
+    X run = 0;
+#pragma unroll
+    for (int j = 0; j < P; ++j) {
+#pragma unroll
+      for (int ww = 0; ww < GW; ++ww) {
+        const X v = r[j * GW + ww];
+        if (ww == G.wig) out[j] = run + w[j];
+        run += v;
+      }
+    }
+    return run;
+  }
 }
 
-// first index i in [0, n) with a[i] >= x (n if none)
+// first index i in [0, n) with a[i] >= x
 __device__ __forceinline__ int lower_bound_u64(const u64* a, int n, u64 x) {
   int lo = 0;
   while (n > 0) {
@@ -185,7 +256,7 @@ __device__ __forceinline__ int lower_bound_u64(const u64* a, int n, u64 x) {
   }
   return lo;
 }
-// first index i in [0, n) with a[i] > x (n if none)
+// first index i in [0, n) with a[i] > x
 __device__ __forceinline__ int upper_bound_u64(const u64* a, int n, u64 x) {
   int lo = 0;
   while (n > 0) {
@@ -201,80 +272,107 @@ __device__ __forceinline__ int upper_bound_u64(const u64* a, int n, u64 x) {
 }
 
 // ---------------------------------------------------------- resampling
-// Shared-memory scratch of the resampler (RWS uses only `scan`).
 struct ResampleSmem {
-  u64* scan;    // [M] RWS: inclusive sums C; Vose: D over L, then E over H
+  u64* scan;    // [M] RWS: inclusive sums C (u32 or u64); Vose: D over L, then E over H
   u64* prob;    // [M] Vose
   int* alias;   // [M] Vose
   int* lists;   // [M] Vose: L ascending then H ascending
 };
 
-// Ancestor of slot `tid` (a8) from its integer weight q (a7) and uniforms.
-// Every thread of the CTA must call it (barriers inside).
-template <int M, int RES>
-__device__ __forceinline__ int resample_slot(uint32_t q, uint32_t Ua, uint32_t Ub, const ResampleSmem& S,
-                                             u64* red, int& rb, u64* prob_out, int* alias_out) {
-  constexpr int NW = M / 32;
-  const int tid = threadIdx.x;
-  u64 Q;
-  const u64 excl = block_excl_scan_u64<NW>(q, red, rb, Q);
-  if (RES == RES_RWS) {
-    // Roulette Wheel Selection (§VI-F): inclusive sums C, draw
-    // c = floor(U Q / 2^32), ancestor = first j with C_j > c (R9).
-    S.scan[tid] = excl + q;
-    __syncthreads();
-    const u64 c = (static_cast<u64>(Ua) * Q) >> 32;
-    int pos = 0;
+// Ancestors anc[P] of the thread's slots (a8) from integer weights q[P]
+// (a7) and uniforms ua/ub (R9–R11).  All threads of the group call it.
+template <class C>
+__device__ __forceinline__ void resample_group(const uint32_t (&q)[C::P], const uint32_t (&ua)[C::P],
+                                               const uint32_t (&ub)[C::P], int (&anc)[C::P],
+                                               const ResampleSmem& S, GroupCtx& G, u64* prob_out,
+                                               int* alias_out) {
+  constexpr int P = C::P, M = C::M;
+  if constexpr (C::RES == RES_RWS) {
+    // Roulette Wheel Selection (§VI-F): C = inclusive sums of q
+    // in slot order, c = floor(U Q / 2^32), ancestor = first j with C_j > c.
+    using X = typename std::conditional<C::SCAN32, uint32_t, u64>::type;
+    X val[P], inc[P];
 #pragma unroll
-    for (int s = M / 2; s >= 1; s >>= 1)
-      if (S.scan[pos + s - 1] <= c) pos += s;
-    return pos;
+    for (int j = 0; j < P; ++j) val[j] = q[j];
+    const X Q = slot_scan_incl<C, X>(val, inc, G);
+    X* Cs = reinterpret_cast<X*>(S.scan);
+#pragma unroll
+    for (int j = 0; j < P; ++j) Cs[C::slot(G.t, j)] = inc[j];
+    gsync<C::GW>(G.g);
+#pragma unroll
+    for (int j = 0; j < P; ++j) {
+      const X c = static_cast<X>((static_cast<u64>(ua[j]) * Q) >> 32);
+      int pos = 0;
+#pragma unroll
+      for (int s = M / 2; s >= 1; s >>= 1)
+        if (Cs[pos + s - 1] <= c) pos += s;
+      anc[j] = pos;
+    }
   } else {
     // Vose's alias method (PAPER.md:18 §IV, :20–22 §VI-F), table by the
-    // closed form of the sequential sweep (R10): a_j = M q_j, small L = {a < Q},
-    // D = inclusive deficits over L, E = inclusive excesses over H.
-    const u64 a = static_cast<u64>(M) * q;
-    const bool small = a < Q;
-    u64 nL, Dtot, Etot;
-    const uint32_t ls = static_cast<uint32_t>(block_excl_scan_u64<NW>(small ? 1ull : 0ull, red, rb, nL));
-    const u64 def = small ? Q - a : 0ull;
-    const u64 exc = small ? 0ull : a - Q;
-    const u64 Dincl = block_excl_scan_u64<NW>(def, red, rb, Dtot) + def;
-    const u64 Eincl = block_excl_scan_u64<NW>(exc, red, rb, Etot) + exc;
-    const int nl = static_cast<int>(nL);
-    const int h = tid - static_cast<int>(ls);
-    if (small) {
-      S.lists[ls] = tid;
-      S.scan[ls] = Dincl;
-    } else {
-      S.lists[nl + h] = tid;
-      S.scan[nl + h] = Eincl;
+    // closed form of the sequential sweep (R10): a_j = M q_j, small L =
+    // {a < Q}, D = inclusive deficits over L, E = inclusive excesses over H.
+    u64 val[P], tmp[P];
+#pragma unroll
+    for (int j = 0; j < P; ++j) val[j] = q[j];
+    const u64 Q = slot_scan_incl<C, u64>(val, tmp, G);
+    u64 a[P];
+    bool small[P];
+    u64 cnt_in[P], cnt[P], def[P], Dinc[P], exc[P], Einc[P];
+#pragma unroll
+    for (int j = 0; j < P; ++j) {
+      a[j] = static_cast<u64>(M) * q[j];
+      small[j] = a[j] < Q;
+      cnt_in[j] = small[j] ? 1ull : 0ull;
+      def[j] = small[j] ? Q - a[j] : 0ull;
+      exc[j] = small[j] ? 0ull : a[j] - Q;
     }
-    __syncthreads();
-    u64 pr;
-    int al;
-    if (small) {
-      pr = a;
-      const int hh = lower_bound_u64(S.scan + nl, M - nl, Dincl - def);
-      al = S.lists[nl + hh];
-    } else if (Eincl < Dtot) {
-      const int ii = upper_bound_u64(S.scan, nl, Eincl);
-      pr = Q + Eincl - S.scan[ii];
-      al = S.lists[nl + h + 1];
-    } else {
-      pr = Q;
-      al = tid;
+    const int nL = static_cast<int>(slot_scan_incl<C, u64>(cnt_in, cnt, G));
+    const u64 Dtot = slot_scan_incl<C, u64>(def, Dinc, G);
+    slot_scan_incl<C, u64>(exc, Einc, G);
+#pragma unroll
+    for (int j = 0; j < P; ++j) {
+      const int s = C::slot(G.t, j);
+      const int ls = static_cast<int>(cnt[j]) - (small[j] ? 1 : 0);   // smalls before s
+      if (small[j]) {
+        S.lists[ls] = s;
+        S.scan[ls] = Dinc[j];
+      } else {
+        S.lists[nL + (s - ls)] = s;
+        S.scan[nL + (s - ls)] = Einc[j];
+      }
     }
-    S.prob[tid] = pr;
-    S.alias[tid] = al;
-    if (prob_out) {
-      prob_out[tid] = pr;
-      alias_out[tid] = al;
+    gsync<C::GW>(G.g);
+#pragma unroll
+    for (int j = 0; j < P; ++j) {
+      const int s = C::slot(G.t, j);
+      const int ls = static_cast<int>(cnt[j]) - (small[j] ? 1 : 0);
+      u64 pr;
+      int al;
+      if (small[j]) {
+        pr = a[j];
+        al = S.lists[nL + lower_bound_u64(S.scan + nL, M - nL, Dinc[j] - def[j])];
+      } else if (Einc[j] < Dtot) {
+        pr = Q + Einc[j] - S.scan[upper_bound_u64(S.scan, nL, Einc[j])];
+        al = S.lists[nL + (s - ls) + 1];
+      } else {
+        pr = Q;
+        al = s;
+      }
+      S.prob[s] = pr;
+      S.alias[s] = al;
+      if (prob_out) {
+        prob_out[s] = pr;
+        alias_out[s] = al;
+      }
     }
-    __syncthreads();
-    const int b = static_cast<int>((static_cast<u64>(Ua) * M) >> 32);
-    const u64 c = (static_cast<u64>(Ub) * Q) >> 32;
-    return c < S.prob[b] ? b : S.alias[b];
+    gsync<C::GW>(G.g);
+#pragma unroll
+    for (int j = 0; j < P; ++j) {
+      const int b = static_cast<int>((static_cast<u64>(ua[j]) * M) >> 32);
+      const u64 c = (static_cast<u64>(ub[j]) * Q) >> 32;
+      anc[j] = c < S.prob[b] ? b : S.alias[b];
+    }
   }
 }
 
@@ -298,207 +396,387 @@ __device__ __forceinline__ long long mailbox_row(const StepParams& P, long long 
   return rq == (r0 - 1 + P.R) % P.R ? P.n_local + cq : P.n_local + P.C + cq;
 }
 
-// ---------------------------------------------------------- smem layout
-template <int NJ, int M, int RES>
-struct StepSmem {
+// ------------------------------------------------------------ sampling
+// Process noise of one particle, Box–Muller pair by pair (R12, R13): pair qp
+// uses Philox words w = 2+2qp, 3+2qp of block w/4; block 0 (words 0–1 = the
+// resampling draw) is supplied by the caller (its words 2, 3 in blk.z/.w).
+struct NoiseGen {
+  uint32_t p, k;
+  const uint32_t (&rk)[20];
+  u32x4 blk;
+  template <int QP>
+  __device__ __forceinline__ void pair(float& z0, float& z1) {
+    constexpr int w = 2 + 2 * QP;
+    if constexpr ((w & 3) == 0) blk = philox4x32_10_rk(p, k, 0u, static_cast<uint32_t>(w >> 2), rk);
+    const uint32_t x0 = (w & 3) == 2 ? blk.z : blk.x;
+    const uint32_t x1 = (w & 3) == 2 ? blk.w : blk.y;
+    normal_pair(x0, x1, z0, z1);
+  }
+};
+
+template <int NJ, int QP>
+struct SamplePairs {
   static constexpr int D = NJ + 4;
-  static constexpr size_t xs = 0;                                  // float [D][M]
-  static constexpr size_t ws = xs + sizeof(float) * D * M;         // float [M]
-  static constexpr size_t scan = ws + sizeof(float) * M;           // u64 [M]
-  static constexpr size_t prob = scan + sizeof(u64) * M;           // u64 [M]   (Vose)
-  static constexpr size_t alias = prob + (RES == RES_VOSE ? sizeof(u64) * M : 0);
-  static constexpr size_t lists = alias + (RES == RES_VOSE ? sizeof(int) * M : 0);
-  static constexpr size_t red = lists + (RES == RES_VOSE ? sizeof(int) * M : 0);   // u64 [2][32]
-  static constexpr size_t misc = red + sizeof(u64) * 64;          // int [128]
-  static constexpr size_t zin = misc + sizeof(int) * 128;         // float [64]: z (NJ+2), h_s u (NJ)
-  static constexpr size_t bar = zin + sizeof(float) * 64;         // mbarrier
-  static constexpr size_t bytes = bar + 16;
+  template <typename X>
+  __device__ __forceinline__ static void run(const ArmConsts& mc, const float* hsu, const X& x, NoiseGen& gen,
+                                             float (&xo)[NJ + 4]) {
+    float z0, z1;
+    gen.template pair<QP>(z0, z1);
+    xo[2 * QP] = arm_sample_comp<NJ, 2 * QP>(mc, hsu, x, z0);
+    if constexpr (2 * QP + 1 < D) xo[2 * QP + 1] = arm_sample_comp<NJ, 2 * QP + 1>(mc, hsu, x, z1);
+    if constexpr (QP + 1 < (D + 1) / 2) SamplePairs<NJ, QP + 1>::run(mc, hsu, x, gen, xo);
+  }
 };
 
 // ------------------------------------------------------------ the kernel
-template <int NJ, int M, int RES>
-__global__ void __launch_bounds__(M) pf_step_kernel(const __grid_constant__ StepParams P) {
-  constexpr int D = NJ + 4;
-  constexpr int E = D + 2;   // mailbox entry: [logw, index bits, x_0..x_{D-1}]
-  constexpr int NW = M / 32;
-  using L = StepSmem<NJ, M, RES>;
+template <class C>
+__global__ void __launch_bounds__(C::T* C::S) pf_step_kernel(const __grid_constant__ StepParams P) {
+  constexpr int NJ = C::NJ, M = C::M, D = C::D, E = C::E, GW = C::GW, PP = C::P;
   extern __shared__ __align__(128) unsigned char smem[];
-  float* xs = reinterpret_cast<float*>(smem + L::xs);
-  float* ws = reinterpret_cast<float*>(smem + L::ws);
-  u64* red = reinterpret_cast<u64*>(smem + L::red);
-  int* misc = reinterpret_cast<int*>(smem + L::misc);
-  float* z_s = reinterpret_cast<float*>(smem + L::zin);
+  float* z_s = reinterpret_cast<float*>(smem + C::c_zin);
   float* hsu_s = z_s + NJ + 2;
-  u64* bar = reinterpret_cast<u64*>(smem + L::bar);
-  ResampleSmem S;
-  S.scan = reinterpret_cast<u64*>(smem + L::scan);
-  S.prob = reinterpret_cast<u64*>(smem + L::prob);
-  S.alias = reinterpret_cast<int*>(smem + L::alias);
-  S.lists = reinterpret_cast<int*>(smem + L::lists);
 
-  const int tid = threadIdx.x;
+  const int g = threadIdx.x / C::T;
+  unsigned char* gs = smem + C::c_groups + g * C::group_bytes;
+  u64* bars = reinterpret_cast<u64*>(gs + C::g_bar);
+  ResampleSmem S;
+  S.scan = reinterpret_cast<u64*>(gs + C::g_scan);
+  S.prob = reinterpret_cast<u64*>(gs + C::g_prob);
+  S.alias = reinterpret_cast<int*>(gs + C::g_alias);
+  S.lists = reinterpret_cast<int*>(gs + C::g_lists);
+  int* anc_s = reinterpret_cast<int*>(gs + C::g_slot);           // STAGED only
+  uint32_t* bz_s = reinterpret_cast<uint32_t*>(anc_s + M);
+  uint32_t* bw_s = bz_s + M;
+  GroupCtx G;
+  G.g = g;
+  G.t = threadIdx.x - g * C::T;
+  G.lane = threadIdx.x & 31;
+  G.wig = G.t >> 5;
+  G.red = reinterpret_cast<u64*>(gs + C::g_red);
+  G.rb = 0;
+  u64* cand = reinterpret_cast<u64*>(gs + C::g_cand);             // [GW][KMAX+1]
+  int* wlist = reinterpret_cast<int*>(gs + C::g_misc) + G.wig * C::KMAX;   // this warp's copy
+
   const int mode = P.mode;
   const bool do_merge = (mode == MODE_EXCHANGE) || (mode == MODE_STEP && !P.first);
   const bool do_resample = (mode == MODE_STEP && !P.first);
   const bool do_sample = (mode == MODE_STEP || mode == MODE_SAMPLE);
   const int K = P.deg * P.t;
+  const long long gid0 = static_cast<long long>(blockIdx.x) * C::S + g;
+  const long long gstride = static_cast<long long>(gridDim.x) * C::S;
 
-  if (tid == 0) {
-    mbar_init(bar, 1);
+  if (G.t == 0) {
+    mbar_init(bars, 1);
+    mbar_init(bars + 1, 1);
     fence_mbar_init();
+    if (gid0 < P.n_local) {
+      mbar_arrive_expect_tx(bars, static_cast<uint32_t>(C::stage_bytes));
+      bulk_g2s(gs + C::g_stage, P.parts + gid0 * C::ROW, static_cast<uint32_t>(C::stage_bytes), bars);
+    }
   }
   if (do_sample) {
-    if (tid < NJ + 2) z_s[tid] = P.z[tid];
-    if (tid < NJ) hsu_s[tid] = P.mc.hs * P.u[tid];
+    if (threadIdx.x < NJ + 2) z_s[threadIdx.x] = P.z[threadIdx.x];
+    if (threadIdx.x < NJ) hsu_s[threadIdx.x] = P.mc.hs * P.u[threadIdx.x];
   }
   __syncthreads();
 
-  int rb = 0;
-  uint32_t parity = 0;
-  for (long long n = blockIdx.x; n < P.n_local; n += gridDim.x) {
-    const long long g = P.g0 + n;
-    const uint32_t pbase = static_cast<uint32_t>(g * M);
-    const uint32_t pidx = pbase + tid;
-    // ---- load the sub-filter's D state rows + log-weight row (TMA bulk)
-    if (tid == 0) {
-      mbar_arrive_expect_tx(bar, (D + 1) * M * sizeof(float));
-#pragma unroll 1
-      for (int c = 0; c < D; ++c) bulk_g2s(xs + c * M, P.state + c * P.stride + n * M, M * sizeof(float), bar);
-      bulk_g2s(ws, P.logw + n * M, M * sizeof(float), bar);
+  int it = 0;
+  for (long long n = gid0; n < P.n_local; n += gstride, ++it) {
+    const int st = (C::NSTAGE == 2) ? (it & 1) : 0;
+    float* xs = reinterpret_cast<float*>(gs + C::g_stage + st * C::stage_bytes);
+    float* ws = xs + D * M;
+    const long long gsf = P.g0 + n;                    // global sub-filter
+    const uint32_t pbase = static_cast<uint32_t>(gsf * M);
+    float* gblk = P.parts + n * C::ROW;                // this sub-filter's block in HBM
+    if constexpr (C::NSTAGE == 2) {   // prefetch the next sub-filter into the other stage
+      if (G.t == 0 && n + gstride < P.n_local) {
+        mbar_arrive_expect_tx(bars + (st ^ 1), static_cast<uint32_t>(C::stage_bytes));
+        bulk_g2s(gs + C::g_stage + (st ^ 1) * C::stage_bytes, P.parts + (n + gstride) * C::ROW,
+                 static_cast<uint32_t>(C::stage_bytes), bars + (st ^ 1));
+      }
+      mbar_wait(bars + st, (it >> 1) & 1);
+    } else {
+      mbar_wait(bars, it & 1);
     }
-    mbar_wait(bar, parity);
-    parity ^= 1;
+
+    float lw[PP];
+#pragma unroll
+    for (int j = 0; j < PP; ++j) lw[j] = ws[C::slot(G.t, j)];
+    uint32_t lmax_o = 0;   // ordered max of the post-exchange log-weights
 
     // ---- a6 exchange: neighbours' best t (mailbox of step k-1) overwrite
     //      the own deg*t worst slots (R2–R5)
     if (do_merge && K > 0) {
-      u64 mk = order_key(ws[tid], static_cast<uint32_t>(tid));
+      // worst K by order key (ascending = worse, R6): per-warp bottom-K by
+      // K rounds of warp REDUX, then a merge of the GW lists after one barrier
+      uint32_t excl = 0;
+      uint32_t wmax = 0;
+#pragma unroll
+      for (int j = 0; j < PP; ++j) wmax = max(wmax, ord_f32(lw[j]));
+      wmax = __reduce_max_sync(0xFFFFFFFFu, wmax);
+      u64 my_cand = ~0ull;
 #pragma unroll 1
       for (int j = 0; j < K; ++j) {
-        const u64 wk = block_min_u64<NW>(mk, red, rb);
+        u64 mk = ~0ull;
+#pragma unroll
+        for (int i = 0; i < PP; ++i) {
+          const u64 key = (excl >> i) & 1u ? ~0ull : order_key(lw[i], static_cast<uint32_t>(C::slot(G.t, i)));
+          mk = key < mk ? key : mk;
+        }
+        const u64 wk = warp_min_u64(mk);
         const int slot = static_cast<int>(0xFFFFFFFFu - static_cast<uint32_t>(wk));
-        if (slot == tid) mk = ~0ull;
-        if (tid == 0) misc[j] = slot;
+#pragma unroll
+        for (int i = 0; i < PP; ++i)
+          if (C::slot(G.t, i) == slot) excl |= 1u << i;
+        if (G.lane == j) my_cand = wk;
       }
-      __syncthreads();
+      if constexpr (GW == 1) {
+        lmax_o = wmax;
+        if (G.lane < K) wlist[G.lane] = static_cast<int>(0xFFFFFFFFu - static_cast<uint32_t>(my_cand));
+      } else {
+        if (G.lane < K) cand[G.wig * (C::KMAX + 1) + G.lane] = my_cand;
+        if (G.lane == 0) cand[G.wig * (C::KMAX + 1) + C::KMAX] = wmax;
+        gsync<GW>(g);
+        // every warp merges the GW candidate lists (identical result in all warps)
+        u64 c[GW];   // candidate i = lane + 32 r of the GW*K list
+        const int ncand = GW * K;
+#pragma unroll
+        for (int r = 0; r < GW; ++r) {
+          const int i = G.lane + 32 * r;
+          c[r] = i < ncand ? cand[(i / K) * (C::KMAX + 1) + i % K] : ~0ull;
+        }
+        uint32_t mo = 0;
+#pragma unroll
+        for (int ww = 0; ww < GW; ++ww) mo = max(mo, static_cast<uint32_t>(cand[ww * (C::KMAX + 1) + C::KMAX]));
+        lmax_o = mo;
+        u64 mine = ~0ull;
 #pragma unroll 1
-      for (int e = tid; e < K * E; e += M) {
+        for (int j = 0; j < K; ++j) {
+          u64 lo = ~0ull;
+#pragma unroll
+          for (int r = 0; r < GW; ++r) lo = c[r] < lo ? c[r] : lo;
+          const u64 wk = warp_min_u64(lo);
+#pragma unroll
+          for (int r = 0; r < GW; ++r)
+            if (c[r] == wk) c[r] = ~0ull;
+          if (G.lane == j) mine = wk;
+        }
+        if (G.lane < K) wlist[G.lane] = static_cast<int>(0xFFFFFFFFu - static_cast<uint32_t>(mine));
+        // own slots among the final worst K
+        excl = 0;
+        __syncwarp();
+#pragma unroll 1
+        for (int j = 0; j < K; ++j) {
+          const int s = wlist[j];
+#pragma unroll
+          for (int i = 0; i < PP; ++i)
+            if (C::slot(G.t, i) == s) excl |= 1u << i;
+        }
+      }
+      __syncwarp();
+#pragma unroll 1
+      for (int e = G.t; e < K * E; e += C::T) {
         const int j = e / E, c = e - j * E;
         const int qi = j / P.t, jj = j - qi * P.t;
-        const long long row = mailbox_row(P, neighbor_of(P, g, qi));
+        const long long row = mailbox_row(P, neighbor_of(P, gsf, qi));
         const float v = P.mb_prev[(row * P.tt + jj) * E + c];
-        const int slot = misc[j];
+        const int slot = wlist[j];
         if (c == 0) ws[slot] = v;
         else if (c >= 2) xs[(c - 2) * M + slot] = v;
       }
       if (P.dbg_src) {
-        long long src = pidx;
+#pragma unroll
+        for (int i = 0; i < PP; ++i) {
+          const int s = C::slot(G.t, i);
+          long long src = pbase + s;
+          if ((excl >> i) & 1u)
 #pragma unroll 1
-        for (int j = 0; j < K; ++j)
-          if (misc[j] == tid) {
-            const int qi = j / P.t, jj = j - qi * P.t;
-            const long long row = mailbox_row(P, neighbor_of(P, g, qi));
-            src = __float_as_uint(P.mb_prev[(row * P.tt + jj) * E + 1]);
-          }
-        P.dbg_src[n * M + tid] = src;
+            for (int j = 0; j < K; ++j)
+              if (wlist[j] == s) {
+                const int qi = j / P.t, jj = j - qi * P.t;
+                const long long row = mailbox_row(P, neighbor_of(P, gsf, qi));
+                src = __float_as_uint(P.mb_prev[(row * P.tt + jj) * E + 1]);
+              }
+          P.dbg_src[n * M + s] = src;
+        }
       }
-      __syncthreads();
+      gsync<GW>(g);
+      // post-exchange max = max(pre-exchange max, incoming): the pre-exchange
+      // maximum value survives because deg*t < m (R19)
+#pragma unroll 1
+      for (int j = 0; j < K; ++j) lmax_o = max(lmax_o, ord_f32(ws[wlist[j]]));
+#pragma unroll
+      for (int j = 0; j < PP; ++j)
+        if ((excl >> j) & 1u) lw[j] = ws[C::slot(G.t, j)];
     } else if ((do_merge || mode == MODE_STEP) && P.dbg_src) {
-      P.dbg_src[n * M + tid] = pidx;   // no exchange (k = 1 or deg*t = 0): identity
+#pragma unroll
+      for (int j = 0; j < PP; ++j) {
+        const int s = C::slot(G.t, j);
+        P.dbg_src[n * M + s] = pbase + s;   // no exchange (k = 1 or deg*t = 0): identity
+      }
     }
 
     if (mode == MODE_EXCHANGE) {
       fence_proxy_async_smem();
-      __syncthreads();
+      gsync<GW>(g);
+      if constexpr (C::NSTAGE == 1) {
+        if (G.t == 0 && n + gstride < P.n_local) {
+          mbar_arrive_expect_tx(bars, static_cast<uint32_t>(C::stage_bytes));
+          bulk_g2s(gs + C::g_stage, P.parts + (n + gstride) * C::ROW, static_cast<uint32_t>(C::stage_bytes), bars);
+        }
+      }
       continue;
     }
 
     // ---- a7 normalise + a8 resample (slot order, R11)
-    int anc = tid;
-    u32x4 b0;
-    bool have_b0 = false;
-    if (do_resample) {
-      const float lw = ws[tid];
-      const uint32_t lmax_o = block_max_u32<NW>(ord_f32(lw), red, rb);
-      const uint32_t q = expq_c(lw - unord_f32(lmax_o));
-      b0 = philox4x32_10(pidx, P.k, 0u, 0u, P.key0, P.key1);
-      have_b0 = true;
-      anc = resample_slot<M, RES>(q, b0.x, b0.y, S, red, rb, nullptr, nullptr);
-      if (P.dbg_anc) P.dbg_anc[n * M + tid] = anc;
-    } else if (mode == MODE_STEP && P.dbg_anc) {
-      P.dbg_anc[n * M + tid] = tid;
+    int anc[PP];
+    uint32_t bz[PP], bw[PP];   // Philox block 0, words 2-3 (first Box–Muller pair)
+    {
+      uint32_t ua[PP], ub[PP], q[PP];
+#pragma unroll
+      for (int j = 0; j < PP; ++j) {
+        const int s = C::slot(G.t, j);
+        anc[j] = s;
+        ua[j] = ub[j] = bz[j] = bw[j] = 0u;
+        if (do_sample || do_resample) {
+          const u32x4 b0 = philox4x32_10_rk(pbase + s, P.k, 0u, 0u, P.rk);
+          ua[j] = b0.x;
+          ub[j] = b0.y;
+          bz[j] = b0.z;
+          bw[j] = b0.w;
+        }
+      }
+      if (do_resample) {
+        if (K == 0) {   // no exchange this step: group max of the loaded set
+          uint32_t mo = 0;
+#pragma unroll
+          for (int j = 0; j < PP; ++j) mo = max(mo, ord_f32(lw[j]));
+          mo = __reduce_max_sync(0xFFFFFFFFu, mo);
+          if constexpr (GW > 1) {
+            uint32_t* r = reinterpret_cast<uint32_t*>(G.red + G.rb * 64);
+            G.rb ^= 1;
+            if (G.lane == 0) r[G.wig] = mo;
+            gsync<GW>(g);
+            mo = __reduce_max_sync(0xFFFFFFFFu, G.lane < GW ? r[G.lane] : 0u);
+          }
+          lmax_o = mo;
+        }
+        const float lmax = unord_f32(lmax_o);
+#pragma unroll
+        for (int j = 0; j < PP; ++j) q[j] = expq_c(lw[j] - lmax);
+        resample_group<C>(q, ua, ub, anc, S, G, nullptr, nullptr);
+      }
+      if (mode == MODE_STEP && P.dbg_anc) {
+#pragma unroll
+        for (int j = 0; j < PP; ++j) P.dbg_anc[n * M + C::slot(G.t, j)] = anc[j];
+      }
+      if constexpr (C::STAGED) {
+#pragma unroll
+        for (int j = 0; j < PP; ++j) {
+          const int s = C::slot(G.t, j);
+          anc_s[s] = anc[j];
+          bz_s[s] = bz[j];
+          bw_s[s] = bw[j];
+        }
+      }
     }
 
-    float lnew;
-    float xo[D];
     if (do_sample) {
-      // ---- a9 gather + a1 RNG + a2 sample + a3 weight
-      float xin[D], xi[D];
+      // ---- a9 gather (smem) + a1 RNG + a2 sample + a3 weight + a10 store,
+      //      one particle at a time (coalesced rows: consecutive threads,
+      //      consecutive slots)
+#pragma unroll C::UNR
+      for (int j = 0; j < PP; ++j) {
+        const int s = C::slot(G.t, j);
+        int a;
+        uint32_t z2, z3;
+        if constexpr (C::STAGED) {
+          a = anc_s[s];
+          z2 = bz_s[s];
+          z3 = bw_s[s];
+        } else {
+          a = anc[j];
+          z2 = bz[j];
+          z3 = bw[j];
+        }
+        const float* xa = xs + a;
+        auto x = [xa](int c) { return xa[c * M]; };
+        float xo[D];
+        NoiseGen gen{pbase + static_cast<uint32_t>(s), P.k, P.rk, u32x4{0u, 0u, z2, z3}};
+        SamplePairs<NJ, 0>::run(P.mc, hsu_s, x, gen, xo);
+        const float l = arm_loglik<NJ>(P.mc, z_s, xo);
+        float* out = gblk + s;
 #pragma unroll
-      for (int c = 0; c < D; ++c) xin[c] = xs[c * M + anc];
-      if (!have_b0) b0 = philox4x32_10(pidx, P.k, 0u, 0u, P.key0, P.key1);
-      u32x4 blk = b0;
-#pragma unroll
-      for (int qp = 0; qp < (D + 1) / 2; ++qp) {
-        const int w = 2 + 2 * qp;
-        if ((w & 3) == 0) blk = philox4x32_10(pidx, P.k, 0u, static_cast<uint32_t>(w >> 2), P.key0, P.key1);
-        const uint32_t x0 = (w & 3) == 2 ? blk.z : blk.x;
-        const uint32_t x1 = (w & 3) == 2 ? blk.w : blk.y;
-        float z0, z1;
-        normal_pair(x0, x1, z0, z1);
-        xi[2 * qp] = z0;
-        if (2 * qp + 1 < D) xi[2 * qp + 1] = z1;
+        for (int c = 0; c < D; ++c) out[c * M] = xo[c];
+        out[D * M] = l;
+        ws[s] = l;   // own slot: read back below by this thread only
       }
-      arm_sample<NJ>(P.mc, hsu_s, xin, xi, xo);
-      lnew = arm_loglik<NJ>(P.mc, z_s, xo);
-      // ---- a10 store (coalesced: consecutive threads, consecutive columns)
-#pragma unroll
-      for (int c = 0; c < D; ++c) P.state[c * P.stride + n * M + tid] = xo[c];
-      P.logw[n * M + tid] = lnew;
-    } else {   // MODE_PUBLISH: the loaded set is the step's weighted set
-      lnew = ws[tid];
-#pragma unroll
-      for (int c = 0; c < D; ++c) xo[c] = xs[c * M + tid];
     }
 
     // ---- a4 local reduce: best t -> mailbox (k&1); a5 global best key
-    u64 key = order_key(lnew, pidx);
-    const int nbest = P.t > 0 ? P.t : 1;
-#pragma unroll 1
-    for (int j = 0; j < nbest; ++j) {
-      const u64 best = block_max_u64<NW>(key, red, rb);
-      if (best == key) {   // unique owner (index is part of the key)
-        if (j < P.t) {
-          float* e = P.mb_cur + (n * P.tt + j) * E;
-          e[0] = lnew;
-          e[1] = __uint_as_float(pidx);
+    {
+      float lnew[PP];
 #pragma unroll
-          for (int c = 0; c < D; ++c) e[2 + c] = xo[c];
+      for (int j = 0; j < PP; ++j) lnew[j] = do_sample ? ws[C::slot(G.t, j)] : lw[j];
+      uint32_t done = 0;
+      const int nbest = P.t > 0 ? P.t : 1;
+#pragma unroll 1
+      for (int jb = 0; jb < nbest; ++jb) {
+        u64 mk = 0ull;
+#pragma unroll
+        for (int j = 0; j < PP; ++j) {
+          const u64 key = (done >> j) & 1u ? 0ull : order_key(lnew[j], pbase + C::slot(G.t, j));
+          mk = key > mk ? key : mk;
         }
-        if (j == 0) atomicMax(P.key_cur, best);
-        key = 0ull;
+        const u64 best = gmax_u64<GW>(mk, G);
+        const int bslot = static_cast<int>(0xFFFFFFFFu - static_cast<uint32_t>(best) - pbase);
+#pragma unroll
+        for (int j = 0; j < PP; ++j) {
+          if (C::slot(G.t, j) == bslot) {   // unique owner
+            done |= 1u << j;
+            if (jb < P.t) {
+              float* e = P.mb_cur + (n * P.tt + jb) * E;
+              e[0] = lnew[j];
+              e[1] = __uint_as_float(pbase + bslot);
+              // own global write (same thread: program order) or the loaded set
+              const float* src = do_sample ? gblk + bslot : xs + bslot;
+#pragma unroll 4
+              for (int c = 0; c < D; ++c) e[2 + c] = src[c * M];
+            }
+            if (jb == 0) atomicMax(P.key_cur, best);
+          }
+        }
       }
     }
     fence_proxy_async_smem();
-    __syncthreads();
+    gsync<GW>(g);
+    if constexpr (C::NSTAGE == 1) {
+      if (G.t == 0 && n + gstride < P.n_local) {
+        mbar_arrive_expect_tx(bars, static_cast<uint32_t>(C::stage_bytes));
+        bulk_g2s(gs + C::g_stage, P.parts + (n + gstride) * C::ROW, static_cast<uint32_t>(C::stage_bytes), bars);
+      }
+    }
   }
 
   // ---- a5: the last CTA to finish copies the winning particle (R6)
   __shared__ unsigned int s_last;
-  if (tid == 0) {
-    __threadfence();
+  __threadfence();
+  __syncthreads();
+  if (threadIdx.x == 0) {
     const unsigned int prev = atomicAdd(P.counter, 1u);
     s_last = (prev == gridDim.x - 1) ? 1u : 0u;
   }
   __syncthreads();
   if (s_last) {
     __threadfence();
+    const int tid = threadIdx.x;
     if (mode != MODE_EXCHANGE) {
       const u64 key = __ldcg(P.key_cur);
       const uint32_t gidx = 0xFFFFFFFFu - static_cast<uint32_t>(key);
       const long long col = static_cast<long long>(gidx) - P.g0 * M;
+      const float* blk = P.parts + (col / M) * C::ROW + (col % M);
       if (tid < D) {
-        const float v = __ldcg(P.state + tid * P.stride + col);
+        const float v = __ldcg(blk + tid * M);
         P.record[4 + tid] = v;
         if (P.est_out) P.est_out[4 + tid] = v;
       }
@@ -525,40 +803,68 @@ __global__ void __launch_bounds__(M) pf_step_kernel(const __grid_constant__ Step
   }
 }
 
-// Resampling test hook: one CTA per row of integer weights, explicit uniforms.
-template <int M, int RES>
-__global__ void __launch_bounds__(M) pf_resample_debug_kernel(const uint32_t* __restrict__ q,
-                                                              const uint32_t* __restrict__ ua,
-                                                              const uint32_t* __restrict__ ub, int* anc,
-                                                              u64* prob, int* alias, long long N) {
-  __shared__ u64 scan[M];
-  __shared__ u64 pr[RES == RES_VOSE ? M : 1];
-  __shared__ int al[RES == RES_VOSE ? M : 1];
-  __shared__ int lists[RES == RES_VOSE ? M : 1];
-  __shared__ u64 red[64];
-  ResampleSmem S{scan, pr, al, lists};
-  int rb = 0;
-  for (long long n = blockIdx.x; n < N; n += gridDim.x) {
-    const long long i = n * M + threadIdx.x;
-    const int a = resample_slot<M, RES>(q[i], ua[i], ub[i], S, red, rb, prob ? prob + n * M : nullptr,
-                                        alias ? alias + n * M : nullptr);
-    anc[i] = a;
-    __syncthreads();
+// Resampling test hook: the step kernel's group resampler on rows of integer
+// weights q [N][M] with explicit uniforms (one group per row).
+template <class C>
+__global__ void __launch_bounds__(C::T* C::S) pf_resample_debug_kernel(const uint32_t* __restrict__ q,
+                                                                        const uint32_t* __restrict__ ua,
+                                                                        const uint32_t* __restrict__ ub, int* anc,
+                                                                        u64* prob, int* alias, long long N) {
+  extern __shared__ __align__(128) unsigned char smem[];
+  const int g = threadIdx.x / C::T;
+  unsigned char* gs = smem + C::c_groups + g * C::group_bytes;
+  ResampleSmem S;
+  S.scan = reinterpret_cast<u64*>(gs + C::g_scan);
+  S.prob = reinterpret_cast<u64*>(gs + C::g_prob);
+  S.alias = reinterpret_cast<int*>(gs + C::g_alias);
+  S.lists = reinterpret_cast<int*>(gs + C::g_lists);
+  GroupCtx G;
+  G.g = g;
+  G.t = threadIdx.x - g * C::T;
+  G.lane = threadIdx.x & 31;
+  G.wig = G.t >> 5;
+  G.red = reinterpret_cast<u64*>(gs + C::g_red);
+  G.rb = 0;
+  for (long long n = static_cast<long long>(blockIdx.x) * C::S + g; n < N;
+       n += static_cast<long long>(gridDim.x) * C::S) {
+    uint32_t qq[C::P], a[C::P], b[C::P];
+    int an[C::P];
+#pragma unroll
+    for (int j = 0; j < C::P; ++j) {
+      const long long i = n * C::M + C::slot(G.t, j);
+      qq[j] = q[i];
+      a[j] = ua[i];
+      b[j] = ub[i];
+    }
+    resample_group<C>(qq, a, b, an, S, G, prob ? prob + n * C::M : nullptr, alias ? alias + n * C::M : nullptr);
+#pragma unroll
+    for (int j = 0; j < C::P; ++j) anc[n * C::M + C::slot(G.t, j)] = an[j];
+    gsync<C::GW>(g);
   }
 }
 
-// Host-side launch helpers (one explicit instantiation set per n_joints TU).
-template <int NJ, int M, int RES>
+// Host-side launch helpers (explicit instantiation sets per n_joints TU).
+template <class C>
 struct StepKernel {
-  static constexpr size_t smem() { return StepSmem<NJ, M, RES>::bytes; }
+  static constexpr size_t smem() { return C::smem; }
   static cudaError_t prepare(int* blocks_per_sm) {
-    cudaError_t e = cudaFuncSetAttribute(pf_step_kernel<NJ, M, RES>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+    cudaError_t e = cudaFuncSetAttribute(pf_step_kernel<C>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                          static_cast<int>(smem()));
+    if (e == cudaSuccess)
+      e = cudaFuncSetAttribute(pf_resample_debug_kernel<C>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                               static_cast<int>(smem()));
     if (e != cudaSuccess) return e;
-    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, pf_step_kernel<NJ, M, RES>, M, smem());
+    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, pf_step_kernel<C>, C::T * C::S, smem());
   }
   static cudaError_t launch(const StepParams& p, int grid, cudaStream_t s) {
-    pf_step_kernel<NJ, M, RES><<<grid, M, smem(), s>>>(p);
+    pf_step_kernel<C><<<grid, C::T * C::S, smem(), s>>>(p);
+    return cudaGetLastError();
+  }
+  static cudaError_t resample_debug(const uint32_t* q, const uint32_t* ua, const uint32_t* ub, int* anc, u64* prob,
+                                    int* alias, long long N, cudaStream_t s) {
+    const long long ctas = (N + C::S - 1) / C::S;
+    pf_resample_debug_kernel<C><<<static_cast<int>(ctas < 4096 ? ctas : 4096), C::T * C::S, smem(), s>>>(
+        q, ua, ub, anc, prob, alias, N);
     return cudaGetLastError();
   }
 };

@@ -1,31 +1,52 @@
-// pf_registry.h — table of compiled pf_step_kernel<NJ, M, RES> instantiations.
+// pf_registry.h — table of compiled pf_step_kernel instantiations.
+//
 // Each pf_inst_nj*.cu translation unit instantiates one n_joints value for
-// every m in {32, ..., 1024} and both resamplers; the runtime looks entries
-// up by (n_joints, m, resampler).
+// every m in {32, ..., 1024} and both resamplers (plus alternative mappings
+// of the hottest configurations).  The runtime takes the FIRST entry that
+// matches (n_joints, m, resampler); PF_VARIANT=<i> in the environment selects
+// the i-th matching entry instead (tuning knob, default 0).
 #pragma once
 #include <cuda_runtime.h>
 
 #include <cstddef>
+#include <cstdint>
 
 namespace pf {
 struct StepParams;
 
 struct KernelEntry {
   int nj, m, res;
+  int gw, s, nstage, unr;   // warps per sub-filter group, groups per CTA, TMA stages, sample unroll
   cudaError_t (*prepare)(int* blocks_per_sm);
   cudaError_t (*launch)(const StepParams& p, int grid, cudaStream_t s);
+  cudaError_t (*resample_debug)(const uint32_t* q, const uint32_t* ua, const uint32_t* ub, int* anc,
+                                unsigned long long* prob, int* alias, long long N, cudaStream_t s);
   size_t smem;
 };
 
 extern const KernelEntry kEntriesNJ2[];
+extern const int kNumEntriesNJ2;
 extern const KernelEntry kEntriesNJ5[];
+extern const int kNumEntriesNJ5;
 extern const KernelEntry kEntriesNJ28[];
-extern const int kNumEntriesPerNJ;
+extern const int kNumEntriesNJ28;
 }  // namespace pf
 
-#define PF_ENTRY(NJ, M, RES) \
-  { NJ, M, RES, &StepKernel<NJ, M, RES>::prepare, &StepKernel<NJ, M, RES>::launch, StepKernel<NJ, M, RES>::smem() }
-#define PF_ENTRIES_FOR(NJ)                                                                                  \
-  PF_ENTRY(NJ, 32, 0), PF_ENTRY(NJ, 32, 1), PF_ENTRY(NJ, 64, 0), PF_ENTRY(NJ, 64, 1), PF_ENTRY(NJ, 128, 0), \
-      PF_ENTRY(NJ, 128, 1), PF_ENTRY(NJ, 256, 0), PF_ENTRY(NJ, 256, 1), PF_ENTRY(NJ, 512, 0),               \
-      PF_ENTRY(NJ, 512, 1), PF_ENTRY(NJ, 1024, 0), PF_ENTRY(NJ, 1024, 1)
+#define PF_ENTRY(NJ, M, RES, GW, S, NST, UNR)                                                             \
+  {NJ,                                                                                                    \
+   M,                                                                                                     \
+   RES,                                                                                                   \
+   GW,                                                                                                    \
+   S,                                                                                                     \
+   NST,                                                                                                   \
+   UNR,                                                                                                   \
+   &StepKernel<KCfg<NJ, M, RES, GW, S, NST, UNR>>::prepare,                                               \
+   &StepKernel<KCfg<NJ, M, RES, GW, S, NST, UNR>>::launch,                                                \
+   &StepKernel<KCfg<NJ, M, RES, GW, S, NST, UNR>>::resample_debug,                                        \
+   StepKernel<KCfg<NJ, M, RES, GW, S, NST, UNR>>::smem()}
+// Default mapping for small states (d <= 12): two particles per thread
+// (rolled per-particle loop), several sub-filters per CTA for small m.
+#define PF_SMALL_D_ENTRIES(NJ, RES)                                                                       \
+  PF_ENTRY(NJ, 32, RES, 1, 8, 2, 1), PF_ENTRY(NJ, 64, RES, 1, 8, 2, 1), PF_ENTRY(NJ, 128, RES, 2, 4, 2, 1), \
+      PF_ENTRY(NJ, 256, RES, 4, 2, 2, 1), PF_ENTRY(NJ, 512, RES, 8, 1, 2, 1),                              \
+      PF_ENTRY(NJ, 1024, RES, 16, 1, 1, 1)

@@ -31,17 +31,37 @@ constexpr size_t kOffMu0 = 512;       // float[64]
 constexpr size_t kOffSigma0 = 768;    // float[64]
 constexpr size_t kScratchBytes = 1024;
 
+struct Table {
+  const pf::KernelEntry* e;
+  int n;
+};
+Table tables(int i) {
+  switch (i) {
+    case 0: return {pf::kEntriesNJ2, pf::kNumEntriesNJ2};
+    case 1: return {pf::kEntriesNJ5, pf::kNumEntriesNJ5};
+    default: return {pf::kEntriesNJ28, pf::kNumEntriesNJ28};
+  }
+}
+
+// First entry matching (nj, m, res), or the PF_VARIANT-th one if set.
 const pf::KernelEntry* find_entry(int nj, int m, int res) {
-  const pf::KernelEntry* tables[] = {pf::kEntriesNJ2, pf::kEntriesNJ5, pf::kEntriesNJ28};
-  for (const pf::KernelEntry* t : tables)
-    for (int i = 0; i < pf::kNumEntriesPerNJ; ++i)
-      if (t[i].nj == nj && t[i].m == m && t[i].res == res) return &t[i];
-  return nullptr;
+  const char* v = std::getenv("PF_VARIANT");
+  int want = v ? std::atoi(v) : 0;
+  const pf::KernelEntry* first = nullptr;
+  for (int ti = 0; ti < 3; ++ti) {
+    const Table t = tables(ti);
+    for (int i = 0; i < t.n; ++i)
+      if (t.e[i].nj == nj && t.e[i].m == m && t.e[i].res == res) {
+        if (!first) first = &t.e[i];
+        if (want-- == 0) return &t.e[i];
+      }
+  }
+  return first;
 }
 
 struct Geometry {
   int nj, d, m, deg, tt, E;
-  long long N, R, C, n_local, g0, n_ext, M_local;
+  long long N, R, C, n_local, g0, n_ext, M_local, ROW;
 };
 
 pf_status validate(const pf_config* cfg, const pf_model_params* mp, Geometry* g) {
@@ -63,7 +83,7 @@ pf_status validate(const pf_config* cfg, const pf_model_params* mp, Geometry* g)
   g->N = cfg->n_filters;
   g->deg = cfg->topo == PF_TOPO_RING ? 2 : cfg->topo == PF_TOPO_TORUS2D ? 4 : 0;
   if (static_cast<long long>(g->deg) * cfg->t >= m && g->deg * cfg->t > 0) return PF_EINVAL;   // R19
-  if (g->deg * cfg->t > 128) return PF_EINVAL;
+  if (g->deg * cfg->t > 32) return PF_EINVAL;   // exchange list fits one warp (KMAX)
   g->tt = cfg->t > 0 ? cfg->t : 1;
   g->E = g->d + 2;
   g->R = g->C = 0;
@@ -90,6 +110,7 @@ pf_status validate(const pf_config* cfg, const pf_model_params* mp, Geometry* g)
     g->n_ext = g->n_local + ((W > 1 && cfg->topo == PF_TOPO_RING) ? 2 : 0);
   }
   g->M_local = g->n_local * m;
+  g->ROW = static_cast<long long>(g->d + 1) * m;
   if (g->M_local > (1ll << 31) || g->N * m > (1ll << 32)) return PF_EINVAL;
   return PF_OK;
 }
@@ -101,8 +122,7 @@ struct pf_handle {
   pf_model_params mp;
   Geometry g;
   pf::ArmConsts mc;
-  float* state;
-  float* logw;
+  float* parts;      // [n_local][d+1][m] blocked SoA (row d = log-weight)
   float* mailbox;
   unsigned char* scratch;
   cudaStream_t stream;
@@ -138,9 +158,7 @@ pf::StepParams base_params(pf_handle* h, long long k, int mode) {
   pf::StepParams p;
   std::memset(&p, 0, sizeof(p));
   p.mc = h->mc;
-  p.state = h->state;
-  p.logw = h->logw;
-  p.stride = h->g.M_local;
+  p.parts = h->parts;
   p.mb_prev = mailbox_parity(h, k - 1);
   p.mb_cur = mailbox_parity(h, k);
   p.z = inputs(h);
@@ -161,8 +179,12 @@ pf::StepParams base_params(pf_handle* h, long long k, int mode) {
   p.tt = h->g.tt;
   p.topo = h->cfg.topo;
   p.deg = h->g.deg;
-  p.key0 = static_cast<uint32_t>(h->cfg.seed);
-  p.key1 = static_cast<uint32_t>(h->cfg.seed >> 32);
+  const uint32_t key0 = static_cast<uint32_t>(h->cfg.seed);
+  const uint32_t key1 = static_cast<uint32_t>(h->cfg.seed >> 32);
+  for (int r = 0; r < 10; ++r) {
+    p.rk[2 * r] = key0 + static_cast<uint32_t>(r) * 0x9E3779B9u;
+    p.rk[2 * r + 1] = key1 + static_cast<uint32_t>(r) * 0xBB67AE85u;
+  }
   p.k = static_cast<uint32_t>(k);
   p.mode = mode;
   p.first = (k == 1) ? 1 : 0;
@@ -187,25 +209,27 @@ pf_status launch(pf_handle* h, const pf::StepParams& p) {
   return sticky(h, h->ke->launch(p, h->grid, h->stream));
 }
 
-__global__ void pf_init_kernel(float* state, float* logw, long long stride, long long M_local, uint32_t p0, int d,
-                               const float* mu0, const float* s0, uint32_t key0, uint32_t key1) {
+__global__ void pf_init_kernel(float* parts, int m, long long M_local, uint32_t p0, int d, const float* mu0,
+                               const float* s0, uint32_t key0, uint32_t key1) {
   // F11: x_c = fma(sigma0_c, xi_c, mu0_c); pair q of particle p from words
   // 2(q&1), 2(q&1)+1 of Philox (p, 0, 2, q>>1) (R13, stream 2 = init).
+  const long long row = static_cast<long long>(d + 1) * m;
   for (long long col = blockIdx.x * static_cast<long long>(blockDim.x) + threadIdx.x; col < M_local;
        col += static_cast<long long>(gridDim.x) * blockDim.x) {
     const uint32_t p = p0 + static_cast<uint32_t>(col);
-    pf::u32x4 blk{0, 0, 0, 0};
+    float* blk = parts + (col / m) * row + (col % m);
+    pf::u32x4 blk4{0, 0, 0, 0};
     for (int q = 0; q < (d + 1) / 2; ++q) {
-      if ((q & 1) == 0) blk = pf::philox4x32_10(p, 0u, 2u, static_cast<uint32_t>(q >> 1), key0, key1);
-      const uint32_t x0 = (q & 1) ? blk.z : blk.x;
-      const uint32_t x1 = (q & 1) ? blk.w : blk.y;
+      if ((q & 1) == 0) blk4 = pf::philox4x32_10(p, 0u, 2u, static_cast<uint32_t>(q >> 1), key0, key1);
+      const uint32_t x0 = (q & 1) ? blk4.z : blk4.x;
+      const uint32_t x1 = (q & 1) ? blk4.w : blk4.y;
       float z0, z1;
       pf::normal_pair(x0, x1, z0, z1);
       const int c = 2 * q;
-      state[c * stride + col] = __fmaf_rn(s0[c], z0, mu0[c]);
-      if (c + 1 < d) state[(c + 1) * stride + col] = __fmaf_rn(s0[c + 1], z1, mu0[c + 1]);
+      blk[c * m] = __fmaf_rn(s0[c], z0, mu0[c]);
+      if (c + 1 < d) blk[(c + 1) * m] = __fmaf_rn(s0[c + 1], z1, mu0[c + 1]);
     }
-    logw[col] = 0.0f;
+    blk[d * m] = 0.0f;
   }
 }
 
@@ -232,32 +256,10 @@ __global__ void pf_reduce_records_kernel(const float* recs, int count, int rec_f
   for (int c = lane; c < rec_floats; c += 32) out[c] = recs[src * rec_floats + c];
 }
 
-template <int M, int RES>
-cudaError_t launch_resample_debug(const uint32_t* q, const uint32_t* ua, const uint32_t* ub, int* anc, u64* prob,
-                                  int* alias, long long N, cudaStream_t s) {
-  const int grid = static_cast<int>(N < 4096 ? N : 4096);
-  pf::pf_resample_debug_kernel<M, RES><<<grid, M, 0, s>>>(q, ua, ub, anc, prob, alias, N);
-  return cudaGetLastError();
-}
-
-cudaError_t resample_debug_dispatch(int m, int res, const uint32_t* q, const uint32_t* ua, const uint32_t* ub,
-                                    int* anc, u64* prob, int* alias, long long N, cudaStream_t s) {
-#define PF_RD(MM)                                                                    \
-  case MM:                                                                           \
-    return res ? launch_resample_debug<MM, 1>(q, ua, ub, anc, prob, alias, N, s) \
-               : launch_resample_debug<MM, 0>(q, ua, ub, anc, prob, alias, N, s);
-  switch (m) {
-    PF_RD(32)
-    PF_RD(64)
-    PF_RD(128)
-    PF_RD(256)
-    PF_RD(512)
-    PF_RD(1024)
-    default:
-      return cudaErrorInvalidValue;
-  }
-#undef PF_RD
-}
+// host [d][M_local] rows <-> device blocked [n_local][d+1][m]: row c of the
+// host array maps to row c of every block (cudaMemcpy2D, pitch = block size).
+cudaError_t rows_to_device(pf_handle* h, const float* host, int row0, int nrows);
+cudaError_t rows_to_host(pf_handle* h, float* host, int row0, int nrows);
 
 template <typename T>
 struct DevBuf {
@@ -270,9 +272,6 @@ struct DevBuf {
 
 }  // namespace
 
-namespace pf {
-const int kNumEntriesPerNJ = 12;
-}
 
 extern "C" {
 
@@ -280,8 +279,7 @@ pf_status pf_query_sizes(const pf_config* cfg, const pf_model_params* model, pf_
   Geometry g;
   const pf_status s = validate(cfg, model, &g);
   if (s != PF_OK || !out) return s != PF_OK ? s : PF_EINVAL;
-  out->state = sizeof(float) * g.d * g.M_local;
-  out->logw = sizeof(float) * g.M_local;
+  out->state = sizeof(float) * g.ROW * g.n_local;
   out->mailbox = sizeof(float) * 2 * g.n_ext * g.tt * g.E;
   out->scratch = kScratchBytes;
   return PF_OK;
@@ -294,7 +292,7 @@ pf_status pf_init(const pf_config* cfg, const pf_model_params* model, const pf_b
   Geometry g;
   pf_status s = validate(cfg, model, &g);
   if (s != PF_OK) return s;
-  if (!buffers->state || !buffers->logw || !buffers->mailbox || !buffers->scratch) return PF_EINVAL;
+  if (!buffers->state || !buffers->mailbox || !buffers->scratch) return PF_EINVAL;
   pf_handle* h = new (std::nothrow) pf_handle();
   if (!h) return PF_ENOMEM;
   h->cfg = *cfg;
@@ -308,8 +306,7 @@ pf_status pf_init(const pf_config* cfg, const pf_model_params* model, const pf_b
   h->mc.s_vel = model->sigma_vel;
   h->mc.inv_cam = 1.0f / model->sigma_cam;
   h->mc.inv_thm = 1.0f / model->sigma_theta_meas;
-  h->state = static_cast<float*>(buffers->state);
-  h->logw = static_cast<float*>(buffers->logw);
+  h->parts = static_cast<float*>(buffers->state);
   h->mailbox = static_cast<float*>(buffers->mailbox);
   h->scratch = static_cast<unsigned char*>(buffers->scratch);
   h->stream = static_cast<cudaStream_t>(cuda_stream);
@@ -342,7 +339,7 @@ pf_status pf_init(const pf_config* cfg, const pf_model_params* model, const pf_b
   if (e == cudaSuccess) {
     const long long blocks = (g.M_local + 255) / 256;
     pf_init_kernel<<<static_cast<int>(blocks < 8 * sms ? blocks : 8 * sms), 256, 0, h->stream>>>(
-        h->state, h->logw, g.M_local, g.M_local, static_cast<uint32_t>(g.g0 * g.m), g.d,
+        h->parts, g.m, g.M_local, static_cast<uint32_t>(g.g0 * g.m), g.d,
         reinterpret_cast<const float*>(h->scratch + kOffMu0), reinterpret_cast<const float*>(h->scratch + kOffSigma0),
         static_cast<uint32_t>(cfg->seed), static_cast<uint32_t>(cfg->seed >> 32));
     e = cudaGetLastError();
@@ -449,9 +446,8 @@ pf_status pf_get_particles(pf_handle* h, float* state_host, float* logw_host, in
   if (h->err != PF_OK) return h->err;
   cudaError_t e = cudaStreamSynchronize(h->stream);
   if (e == cudaSuccess)
-    e = cudaMemcpy(state_host, h->state, sizeof(float) * h->g.d * h->g.M_local, cudaMemcpyDeviceToHost);
-  if (e == cudaSuccess && logw_host)
-    e = cudaMemcpy(logw_host, h->logw, sizeof(float) * h->g.M_local, cudaMemcpyDeviceToHost);
+    e = rows_to_host(h, state_host, 0, h->g.d);
+  if (e == cudaSuccess && logw_host) e = rows_to_host(h, logw_host, h->g.d, 1);
   if (step) *step = h->step;
   return sticky(h, e);
 }
@@ -468,8 +464,8 @@ pf_status pf_set_particles(pf_handle* h, const float* state_host, const float* l
   if (h->err != PF_OK) return h->err;
   cudaError_t e = cudaStreamSynchronize(h->stream);
   if (e == cudaSuccess)
-    e = cudaMemcpy(h->state, state_host, sizeof(float) * h->g.d * h->g.M_local, cudaMemcpyHostToDevice);
-  if (e == cudaSuccess) e = cudaMemcpy(h->logw, logw_host, sizeof(float) * h->g.M_local, cudaMemcpyHostToDevice);
+    e = rows_to_device(h, state_host, 0, h->g.d);
+  if (e == cudaSuccess) e = rows_to_device(h, logw_host, h->g.d, 1);
   if (e != cudaSuccess) return sticky(h, e);
   pf_status s = publish(h, step);
   if (s != PF_OK) return s;
@@ -484,7 +480,7 @@ pf_status pf_debug_sample_weight(pf_handle* h, const float* state_in, const floa
   if (h->cfg.world != 1) return PF_ESTATE;
   cudaError_t e = cudaStreamSynchronize(h->stream);
   if (e == cudaSuccess)
-    e = cudaMemcpy(h->state, state_in, sizeof(float) * h->g.d * h->g.M_local, cudaMemcpyHostToDevice);
+    e = rows_to_device(h, state_in, 0, h->g.d);
   if (e == cudaSuccess) e = cudaMemsetAsync(keys(h), 0, 2 * sizeof(u64), h->stream);
   if (e != cudaSuccess) return sticky(h, e);
   pf_status s = stage_inputs(h, z_k, u_km1);
@@ -495,8 +491,8 @@ pf_status pf_debug_sample_weight(pf_handle* h, const float* state_in, const floa
   h->step = k;
   e = cudaStreamSynchronize(h->stream);
   if (e == cudaSuccess)
-    e = cudaMemcpy(state_out, h->state, sizeof(float) * h->g.d * h->g.M_local, cudaMemcpyDeviceToHost);
-  if (e == cudaSuccess) e = cudaMemcpy(logw_out, h->logw, sizeof(float) * h->g.M_local, cudaMemcpyDeviceToHost);
+    e = rows_to_host(h, state_out, 0, h->g.d);
+  if (e == cudaSuccess) e = rows_to_host(h, logw_out, h->g.d, 1);
   return sticky(h, e);
 }
 
@@ -520,8 +516,8 @@ pf_status pf_debug_resample(pf_handle* h, const uint32_t* q, const uint32_t* ua,
   if (e == cudaSuccess) e = cudaMemcpy(dua.p, ua, 4 * n, cudaMemcpyHostToDevice);
   if (e == cudaSuccess) e = cudaMemcpy(dub.p, ub, 4 * n, cudaMemcpyHostToDevice);
   if (e == cudaSuccess)
-    e = resample_debug_dispatch(h->g.m, vose ? 1 : 0, dq.p, dua.p, dub.p, danc.p, want_table ? dpr.p : nullptr,
-                                want_table ? dal.p : nullptr, h->g.N, h->stream);
+    e = h->ke->resample_debug(dq.p, dua.p, dub.p, danc.p, want_table ? dpr.p : nullptr, want_table ? dal.p : nullptr,
+                              h->g.N, h->stream);
   if (e == cudaSuccess) e = cudaStreamSynchronize(h->stream);
   if (e == cudaSuccess) e = cudaMemcpy(ancestors, danc.p, 4 * n, cudaMemcpyDeviceToHost);
   if (e == cudaSuccess && want_table) e = cudaMemcpy(prob, dpr.p, 8 * n, cudaMemcpyDeviceToHost);
@@ -537,7 +533,7 @@ pf_status pf_debug_exchange(pf_handle* h, const float* logw, int64_t* src) {
   DevBuf<long long> dsrc;
   cudaError_t e = dsrc.alloc(M);
   if (e == cudaSuccess) e = cudaStreamSynchronize(h->stream);
-  if (e == cudaSuccess) e = cudaMemcpy(h->logw, logw, sizeof(float) * M, cudaMemcpyHostToDevice);
+  if (e == cudaSuccess) e = rows_to_device(h, logw, h->g.d, 1);
   if (e != cudaSuccess) return sticky(h, e);
   const long long s = h->step > 0 ? h->step : 1;
   pf_status st = publish(h, s);
@@ -609,18 +605,44 @@ const char* pf_strerror(pf_status s) {
 pf_status pf_last_error(const pf_handle* h) { return h ? h->err : PF_EINVAL; }
 
 int32_t pf_supported(int32_t* n_joints, int32_t* m, int32_t cap) {
-  const pf::KernelEntry* tables[] = {pf::kEntriesNJ2, pf::kEntriesNJ5, pf::kEntriesNJ28};
   int32_t n = 0;
-  for (const pf::KernelEntry* t : tables)
-    for (int i = 0; i < pf::kNumEntriesPerNJ; ++i)
-      if (t[i].res == 0) {
-        if (n < cap && n_joints && m) {
-          n_joints[n] = t[i].nj;
-          m[n] = t[i].m;
-        }
-        ++n;
+  for (int ti = 0; ti < 3; ++ti) {
+    const Table t = tables(ti);
+    for (int i = 0; i < t.n; ++i) {
+      bool dup = false;
+      for (int j = 0; j < i; ++j) dup = dup || (t.e[j].m == t.e[i].m && t.e[j].nj == t.e[i].nj);
+      if (t.e[i].res != 0 || dup) continue;
+      if (n < cap && n_joints && m) {
+        n_joints[n] = t.e[i].nj;
+        m[n] = t.e[i].m;
       }
+      ++n;
+    }
+  }
   return n;
 }
 
 }  // extern "C"
+
+namespace {
+cudaError_t rows_to_device(pf_handle* h, const float* host, int row0, int nrows) {
+  const size_t m = h->g.m;
+  for (int r = 0; r < nrows; ++r) {
+    cudaError_t e = cudaMemcpy2D(h->parts + (row0 + r) * m, sizeof(float) * h->g.ROW,
+                                 host + static_cast<size_t>(r) * h->g.M_local, sizeof(float) * m, sizeof(float) * m,
+                                 h->g.n_local, cudaMemcpyHostToDevice);
+    if (e != cudaSuccess) return e;
+  }
+  return cudaSuccess;
+}
+cudaError_t rows_to_host(pf_handle* h, float* host, int row0, int nrows) {
+  const size_t m = h->g.m;
+  for (int r = 0; r < nrows; ++r) {
+    cudaError_t e = cudaMemcpy2D(host + static_cast<size_t>(r) * h->g.M_local, sizeof(float) * m,
+                                 h->parts + (row0 + r) * m, sizeof(float) * h->g.ROW, sizeof(float) * m,
+                                 h->g.n_local, cudaMemcpyDeviceToHost);
+    if (e != cudaSuccess) return e;
+  }
+  return cudaSuccess;
+}
+}  // namespace

@@ -69,12 +69,10 @@ class ParticleFilter:
         with torch.cuda.device(self.device):
             self.stream = stream or torch.cuda.current_stream(self.device)
             alloc = lambda n: torch.empty(max(int(n), 16), dtype=torch.uint8, device=self.device)
-            self._state = alloc(sizes.state)
-            self._logw = alloc(sizes.logw)
+            self._parts = alloc(sizes.state)
             self._mailbox = alloc(sizes.mailbox)
             self._scratch = alloc(sizes.scratch)
-            bufs = B.pf_buffers(self._state.data_ptr(), self._logw.data_ptr(), self._mailbox.data_ptr(),
-                                self._scratch.data_ptr())
+            bufs = B.pf_buffers(self._parts.data_ptr(), self._mailbox.data_ptr(), self._scratch.data_ptr())
             self.h = B.pf_init(self.cfg, mc, bufs, self.stream.cuda_stream, _f32(mu0), _f32(sigma0))
         self.shard = B.pf_get_shard(self.h)
         self.M_local = self.shard.n_local * m
@@ -82,12 +80,10 @@ class ParticleFilter:
 
     # -- views of the caller-owned buffers (torch, device) -------------------
     @property
-    def state(self) -> torch.Tensor:
-        return self._state[: 4 * self.d * self.M_local].view(torch.float32).view(self.d, self.M_local)
-
-    @property
-    def logw(self) -> torch.Tensor:
-        return self._logw[: 4 * self.M_local].view(torch.float32)
+    def particles(self) -> torch.Tensor:
+        """Device particle blocks [n_local][d+1][m] (rows 0..d-1 state, row d log-weight)."""
+        n = self.shard.n_local * (self.d + 1) * self.m
+        return self._parts[: 4 * n].view(torch.float32).view(self.shard.n_local, self.d + 1, self.m)
 
     @property
     def mailbox(self) -> torch.Tensor:

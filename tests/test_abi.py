@@ -59,11 +59,11 @@ def _model(B, nj=2):
 def test_query_sizes(B):
     s = B.pf_query_sizes(_cfg(B), _model(B, 2))
     d, M = 6, 16 * 64
-    assert s.state == 4 * d * M and s.logw == 4 * M
+    assert s.state == 4 * (d + 1) * M          # blocked [n][d+1][m]: states + log-weights
     assert s.mailbox == 4 * 2 * 16 * 1 * (d + 2)
     # sharded ring: 2 halo rows
     s2 = B.pf_query_sizes(_cfg(B, world=4, rank=1, t=2), _model(B, 5))
-    assert s2.state == 4 * 9 * 4 * 64
+    assert s2.state == 4 * 10 * 4 * 64
     assert s2.mailbox == 4 * 2 * (4 + 2) * 2 * 11
 
 

@@ -1,0 +1,110 @@
+"""Multi-rank host logic on CPU (gloo, world_size 2..4): the halo plan and
+its exchange fill every halo row with the right neighbour sub-filter's
+mailbox entries (Alg.2 l.10–14; sharding SURVEY §8(e)), and the
+per-rank estimate records reduce to the oracle's global argmax (R6)."""
+import os
+import socket
+
+import numpy as np
+import pytest
+import torch
+import torch.distributed as dist
+import torch.multiprocessing as mp
+
+from paper_conf_ipps_chitchianasks13_b200 import distributed as Dd
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def _expected_halo_ids(topo, N, world, rank, R=0, C=0):
+    g0, n_local, n_ext = Dd.shard_geometry(topo, N, world, rank, R, C)
+    if topo == "ring":
+        return {n_local: (g0 - 1) % N, n_local + 1: (g0 + n_local) % N}
+    R, C = Dd.torus_shape(N, R, C)
+    r0, rows = g0 // C, n_local // C
+    out = {}
+    for c in range(C):
+        out[n_local + c] = ((r0 - 1) % R) * C + c
+        out[n_local + C + c] = ((r0 + rows) % R) * C + c
+    return out
+
+
+def _worker(rank, world, port, cases, ret):
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        for topo, N, t, E in cases:
+            g0, n_local, n_ext = Dd.shard_geometry(topo, N, world, rank)
+            mb = torch.full((n_ext, t, E), -1.0)
+            for row in range(n_local):
+                mb[row] = float(g0 + row)          # entry = global sub-filter id
+            plan = Dd.halo_plan(topo, N, world)
+            Dd.exchange_halos(mb, plan, rank)
+            for row, gid in _expected_halo_ids(topo, N, world, rank).items():
+                assert torch.all(mb[row] == float(gid)), (topo, N, rank, row, gid, mb[row].flatten()[:3])
+            for row in range(n_local):
+                assert torch.all(mb[row] == float(g0 + row))
+        # estimate protocol: ordered key of every rank's best, all-gather, max
+        rng = np.random.default_rng(7)
+        w = np.round(rng.normal(-20, 5, 64 * world) * 2).astype(np.float32) / 2   # ties across ranks
+        lo = rank * 64
+        mine = w[lo:lo + 64]
+
+        def key(v, p):
+            b = np.array([v], np.float32).view(np.uint32)[0]
+            o = (~b & 0xFFFFFFFF) if b & 0x80000000 else (b | 0x80000000)
+            return (int(o) << 32) | (0xFFFFFFFF - p)
+
+        best = max(key(v, lo + i) for i, v in enumerate(mine))
+        keys = torch.zeros(world, dtype=torch.float64)
+        out = [torch.zeros(2, dtype=torch.int64) for _ in range(world)]
+        dist.all_gather(out, torch.tensor([best >> 32, best & 0xFFFFFFFF], dtype=torch.int64))
+        win = max((int(a) << 32) | int(b) for a, b in out)
+        idx = 0xFFFFFFFF - (win & 0xFFFFFFFF)
+        ref = max(range(len(w)), key=lambda p: (w[p], -p))
+        assert idx == ref
+        ret[rank] = True
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world", [2, 3, 4])
+def test_halo_exchange_gloo(world):
+    cases = [("ring", 4 * world, 1, 11), ("ring", world, 2, 8)]
+    if world in (2, 4):
+        cases += [("torus", 16, 1, 11), ("torus", 64, 2, 6)]
+    ctx = mp.get_context("spawn")
+    ret = ctx.Manager().dict()
+    mp.start_processes(_worker, args=(world, _free_port(), cases, ret), nprocs=world, join=True,
+                       start_method="spawn")
+    assert len(ret) == world
+
+
+def test_loopback_matches_plan():
+    # the single-process loopback applies the same plan
+    for topo, N, world in [("ring", 8, 2), ("ring", 12, 4), ("torus", 16, 2), ("torus", 64, 4)]:
+        mbs = []
+        for r in range(world):
+            g0, n_local, n_ext = Dd.shard_geometry(topo, N, world, r)
+            mb = torch.full((n_ext, 1, 3), -1.0)
+            mb[:n_local] = torch.arange(g0, g0 + n_local, dtype=torch.float32)[:, None, None]
+            mbs.append(mb)
+        Dd.loopback_exchange(mbs, Dd.halo_plan(topo, N, world))
+        for r in range(world):
+            for row, gid in _expected_halo_ids(topo, N, world, r).items():
+                assert torch.all(mbs[r][row] == float(gid))
+
+
+def test_plan_shapes():
+    assert Dd.halo_plan("ring", 8, 1) == []
+    assert Dd.halo_plan("none", 8, 4) == []
+    p = Dd.halo_plan("torus", 64, 4)      # R = C = 8, 2 grid rows per rank
+    assert len(p) == 8 and all(t.nrows == 8 for t in p)
+    assert Dd.shard_geometry("torus", 64, 4, 3) == (48, 16, 32)
+    assert Dd.shard_geometry("ring", 64, 4, 1) == (16, 16, 18)

@@ -185,3 +185,36 @@ def test_step_batch_matches_streaming(P, W):
         x, lw, idx = a.estimate()
         np.testing.assert_array_equal(est[k - 1, 4:].cpu().numpy(), x)
         assert est[k - 1, 2].item() == lw
+
+
+@pytest.mark.parametrize("topo,N,world", [("ring", 16, 2), ("torus", 16, 2), ("ring", 12, 4), ("torus", 64, 4)])
+def test_sharded_loopback_bit_identical(P, orc, W, topo, N, world):
+    # world shards of one filter in one process on one GPU, halos exchanged
+    # by the same plan the NCCL path uses: identical to the unsharded filter
+    # and to the oracle (global Philox counters, exact max reduce)
+    import torch
+    from paper_conf_ipps_chitchianasks13_b200 import distributed as Dd
+    nj, m, T = 5, 64, 6
+    tr = W.make_trajectory(nj, T, 4)
+    kw = dict(m=m, n_filters=N, t=1, topo=topo, resampler="vose", seed=99)
+    shards = [P.ParticleFilter(tr["mu0"], tr["sigma0"], P.ArmModel(n_joints=nj), rank=r, world=world, **kw)
+              for r in range(world)]
+    o = orc.Filter(orc.Config(m=m, n_filters=N, t=1, topo=topo, resampler="vose", seed=99),
+                   orc.Model(n_joints=nj), tr["mu0"], tr["sigma0"])
+    plan = Dd.halo_plan(topo, N, world)
+    recs = torch.zeros(world, 4 + nj + 4, device="cuda")
+    for k in range(1, T + 1):
+        if k > 1:
+            Dd.loopback_exchange([s.mailbox[(k - 1) & 1] for s in shards], plan)
+        for s in shards:
+            s.step(tr["Z"][k], tr["U"][k - 1])
+        for r, s in enumerate(shards):
+            recs[r] = s.record
+        shards[0].reduce_records(recs)
+        o.step(tr["Z"][k], tr["U"][k - 1])
+        xg, lg, ig = shards[0].estimate()
+        xo, lo, io = o.estimate()
+        assert ig == io and np.array_equal(xg, xo), k
+    so, wo, _ = o.get()
+    sg = np.concatenate([s.get_particles()[0] for s in shards], axis=1)
+    np.testing.assert_array_equal(sg, so)
