@@ -209,6 +209,22 @@ pf_status pf_debug_exchange(pf_handle* h, const float* logw, int64_t* src);
 pf_status pf_set_trace(pf_handle* h, int32_t enable);
 pf_status pf_get_trace(pf_handle* h, int64_t* src, int32_t* ancestors);
 
+/* Element-wise evaluation of the device fp32 contract for
+ * bit-exact comparison with the oracle.  Host arrays of 32-bit words:
+ *   PF_MATH_SIN / COS / LOG / SQRT: in float[n] -> out float[n]  (F5, F6, sqrt of F2)
+ *   PF_MATH_EXPQ: in float[n] (delta <= 0) -> out uint32[n]      (F7)
+ *   PF_MATH_SINCOS2PI: in uint32 m23[n] -> out float[2n] (sin, cos)  (F3)
+ *   PF_MATH_NORMAL_PAIR: in uint32 [x0[n], x1[n]] -> out float[2n] (z0, z1)  (F2)
+ *   PF_MATH_PHILOX: in uint32 [c0[n], c1[n], c2[n], c3[n], k0, k1] -> out uint32[4n]  (R12)
+ * No handle; uses the current CUDA device; synchronous. */
+enum { PF_MATH_SIN = 0, PF_MATH_COS = 1, PF_MATH_LOG = 2, PF_MATH_EXPQ = 3, PF_MATH_SQRT = 4,
+       PF_MATH_SINCOS2PI = 5, PF_MATH_NORMAL_PAIR = 6, PF_MATH_PHILOX = 7 };
+pf_status pf_debug_math(int32_t fn, const uint32_t* in, uint32_t* out, int64_t n);
+
+/* Count the float bit patterns x in [lo_bits, hi_bits] for which the
+ * kernels' branch-free sqrt differs from IEEE sqrt.rn (exhaustive, on device). */
+pf_status pf_debug_check_sqrt(uint32_t lo_bits, uint32_t hi_bits, uint64_t* mismatches);
+
 /* Release host metadata; NULL-safe.  Does not free caller buffers. */
 pf_status pf_destroy(pf_handle* h);
 

@@ -23,8 +23,9 @@ ENTRY_POINTS = [
     "pf_query_sizes", "pf_init", "pf_step", "pf_step_batch", "pf_estimate", "pf_record_ptr",
     "pf_reduce_records", "pf_get_shard", "pf_get_particles", "pf_set_particles", "pf_debug_sample_weight",
     "pf_debug_resample", "pf_debug_exchange", "pf_set_trace", "pf_get_trace", "pf_destroy", "pf_strerror",
-    "pf_last_error", "pf_supported",
+    "pf_last_error", "pf_supported", "pf_debug_math", "pf_debug_check_sqrt",
 ]
+PF_MATH = {"sin": 0, "cos": 1, "log": 2, "expq": 3, "sqrt": 4, "sincos2pi": 5, "normal_pair": 6, "philox": 7}
 
 
 class pf_model_params(C.Structure):
@@ -96,6 +97,10 @@ def lib() -> C.CDLL:
         L.pf_strerror.restype = C.c_char_p
         L.pf_supported.argtypes = [P, P, I32]
         L.pf_supported.restype = I32
+        L.pf_debug_math.argtypes = [I32, P, P, I64]
+        L.pf_debug_math.restype = ST
+        L.pf_debug_check_sqrt.argtypes = [C.c_uint32, C.c_uint32, P]
+        L.pf_debug_check_sqrt.restype = ST
         _lib = L
     return _lib
 
@@ -210,3 +215,20 @@ def pf_supported() -> list[tuple[int, int]]:
     m = (C.c_int32 * n)()
     lib().pf_supported(nj, m, n)
     return list(zip(list(nj), list(m)))
+
+
+def pf_debug_math(fn: str, words, n: int):
+    """Evaluate a contract function on the device; words: uint32 numpy array."""
+    import numpy as np
+    k = PF_MATH[fn]
+    w = np.ascontiguousarray(words, dtype=np.uint32)
+    out_n = 2 * n if fn in ("sincos2pi", "normal_pair") else 4 * n if fn == "philox" else n
+    out = np.zeros(max(out_n, 1), np.uint32)
+    check(lib().pf_debug_math(k, w.ctypes.data, out.ctypes.data, n), "pf_debug_math")
+    return out[:out_n]
+
+
+def pf_debug_check_sqrt(lo_bits: int, hi_bits: int) -> int:
+    bad = C.c_uint64()
+    check(lib().pf_debug_check_sqrt(lo_bits, hi_bits, C.byref(bad)), "pf_debug_check_sqrt")
+    return bad.value

@@ -126,7 +126,7 @@ def test_sample_noise_layout(orc, W):
         ref = []
         for q in range(5):
             x0, x1 = int(w[2 + 2 * q]), int(w[3 + 2 * q])
-            u1 = 1 - (x0 >> 9) * 2.0**-23
+            u1 = 1 - ((x0 >> 9) + 0.5) * 2.0**-23
             u2 = (x1 >> 9) * 2.0**-23
             r = math.sqrt(-2 * math.log(u1))
             ref += [r * math.cos(2 * math.pi * u2), r * math.sin(2 * math.pi * u2)]

@@ -53,7 +53,7 @@ def _words(n, seed):
 def test_normal_pair_fp32_vs_fp64(orc):
     # the fp32 contract (F2) agrees with libm double Box–Muller within 1e-5
     w = _words(20000, 1)
-    # include the extreme u1 = 2^-23 (r = 5.64) and u1 = 1 (r = 0)
+    # include the extremes u1 = 2^-24 (r = 5.77) and u1 = 1 - 2^-24 (r = 3.5e-4)
     w[0] = [0xFFFFFFFF, 0x12345678]
     w[1] = [0x000001FF, 0x9ABCDEF0]
     err = 0.0
