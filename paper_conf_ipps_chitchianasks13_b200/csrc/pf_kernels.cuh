@@ -52,6 +52,7 @@ struct StepParams {
   u64* key_cur;            // global best key of this step (0 on entry)
   u64* key_next;           // reset to 0 for the next step
   unsigned int* counter;   // CTA completion counter (0 on entry, reset by the last CTA)
+  unsigned int* work;      // dynamic sub-filter counter (0 on entry, reset by the last CTA)
   float* record;           // [4 + d] estimate record of this shard
   float* est_out;          // nullable [4 + d] (batched mode)
   long long* dbg_src;      // nullable [M_local] exchange sources (global index)
@@ -87,6 +88,9 @@ __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t by
       "l"(src), "r"(bytes), "r"(smem_u32(bar))
       : "memory");
 }
+__device__ __forceinline__ void mbar_arrive(u64* bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
 __device__ __forceinline__ void mbar_wait(u64* bar, uint32_t parity) {
   asm volatile(
       "{\n\t.reg .pred p;\n"
@@ -103,9 +107,10 @@ __device__ __forceinline__ void mbar_wait(u64* bar, uint32_t parity) {
 // group; the per-particle sample/weight loop over a thread's P slots is
 // unrolled UNR times (P for full unrolling; 1 keeps one copy of the
 // ~10–40 KB per-particle code in the instruction cache).
-template <int NJ_, int M_, int RES_, int GW_, int S_, int NSTAGE_, int UNR_>
+template <int NJ_, int M_, int RES_, int GW_, int S_, int NSTAGE_, int UNR_, int MINB_>
 struct KCfg {
   static constexpr int NJ = NJ_, M = M_, RES = RES_, GW = GW_, S = S_, NSTAGE = NSTAGE_, UNR = UNR_;
+  static constexpr int MINB = MINB_;         // __launch_bounds__ min CTAs per SM (register cap)
   static constexpr int D = NJ + 4;
   static constexpr int E = D + 2;            // mailbox entry: [logw, index bits, x_0..x_{D-1}]
   static constexpr int T = 32 * GW;          // threads per group
@@ -120,16 +125,16 @@ struct KCfg {
   // per-group shared memory
   static constexpr size_t stage_bytes = sizeof(float) * ROW;
   static constexpr size_t g_stage = 0;
-  static constexpr size_t g_scan = NSTAGE * stage_bytes;                          // u64 [M]
-  static constexpr size_t g_slot = g_scan + sizeof(u64) * M;                      // int anc[M], u32 bz[M], bw[M]
-  static constexpr size_t g_prob = g_slot + (STAGED ? 12 * M : 0);                // u64 [M]  (Vose)
+  static constexpr size_t g_scan = NSTAGE * stage_bytes;                          // u64 [M]; after the
+                                                                                  // resample: Philox words
+  static constexpr size_t g_prob = g_scan + sizeof(u64) * M;                      // u64 [M]  (Vose)
   static constexpr size_t g_alias = g_prob + (RES == RES_VOSE ? sizeof(u64) * M : 0);
   static constexpr size_t g_lists = g_alias + (RES == RES_VOSE ? sizeof(int) * M : 0);
-  static constexpr size_t g_red = g_lists + (RES == RES_VOSE ? sizeof(int) * M : 0);   // u64 [2][64]
-  static constexpr size_t g_cand = g_red + sizeof(u64) * 128;                    // u64 [GW][KMAX+1]
+  static constexpr size_t g_red = g_lists + (RES == RES_VOSE ? sizeof(int) * M : 0);   // u64 [2][32]
+  static constexpr size_t g_cand = g_red + sizeof(u64) * 64;                     // u64 [GW][KMAX+1]
   static constexpr size_t g_misc = g_cand + sizeof(u64) * GW * (KMAX + 1);       // int [GW][KMAX]
-  static constexpr size_t g_bar = g_misc + sizeof(int) * GW * KMAX;              // u64 [2]
-  static constexpr size_t group_bytes = (g_bar + 16 + 127) / 128 * 128;
+  static constexpr size_t g_bar = g_misc + sizeof(int) * GW * KMAX;              // u64 [2] + next [2]
+  static constexpr size_t group_bytes = (g_bar + 32 + 127) / 128 * 128;
   // per-CTA
   static constexpr size_t c_zin = 0;          // float [64]: z (NJ+2), h_s u (NJ)
   static constexpr size_t c_groups = 256;
@@ -153,7 +158,7 @@ struct GroupCtx {
   int g;          // group index in the CTA
   int t;          // thread index in the group
   int lane, wig;  // lane, warp in group
-  u64* red;       // [2][64] cross-warp reduction slots
+  u64* red;       // [2][32] cross-warp reduction slots
   int rb;         // slot toggle (uniform in the group); each call with GW > 1
                   // syncs once, so a slot is reusable two calls later
 };
@@ -177,7 +182,7 @@ __device__ __forceinline__ u64 gmax_u64(u64 v, GroupCtx& G) {
   if constexpr (GW == 1) {
     return w;
   } else {
-    u64* r = G.red + G.rb * 64;
+    u64* r = G.red + G.rb * 32;
     G.rb ^= 1;
     if (G.lane == 0) r[G.wig] = w;
     gsync<GW>(G.g);
@@ -221,7 +226,7 @@ __device__ __forceinline__ X slot_scan_incl(const X (&val)[C::P], X (&out)[C::P]
     }
     return base;
   } else {
-    X* r = reinterpret_cast<X*>(G.red + G.rb * 64);
+    X* r = reinterpret_cast<X*>(G.red + G.rb * 32);
     G.rb ^= 1;
     if (G.lane == 31) {
 #pragma unroll
@@ -430,7 +435,7 @@ struct SamplePairs {
 
 // ------------------------------------------------------------ the kernel
 template <class C>
-__global__ void __launch_bounds__(C::T* C::S) pf_step_kernel(const __grid_constant__ StepParams P) {
+__global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __grid_constant__ StepParams P) {
   constexpr int NJ = C::NJ, M = C::M, D = C::D, E = C::E, GW = C::GW, PP = C::P;
   extern __shared__ __align__(128) unsigned char smem[];
   float* z_s = reinterpret_cast<float*>(smem + C::c_zin);
@@ -444,9 +449,8 @@ __global__ void __launch_bounds__(C::T* C::S) pf_step_kernel(const __grid_consta
   S.prob = reinterpret_cast<u64*>(gs + C::g_prob);
   S.alias = reinterpret_cast<int*>(gs + C::g_alias);
   S.lists = reinterpret_cast<int*>(gs + C::g_lists);
-  int* anc_s = reinterpret_cast<int*>(gs + C::g_slot);           // STAGED only
-  uint32_t* bz_s = reinterpret_cast<uint32_t*>(anc_s + M);
-  uint32_t* bw_s = bz_s + M;
+  uint2* bzw_s = reinterpret_cast<uint2*>(gs + C::g_scan);       // STAGED: Philox words after the resample
+  volatile unsigned int* next_s = reinterpret_cast<unsigned int*>(gs + C::g_bar + 16);
   GroupCtx G;
   G.g = g;
   G.t = threadIdx.x - g * C::T;
@@ -465,14 +469,28 @@ __global__ void __launch_bounds__(C::T* C::S) pf_step_kernel(const __grid_consta
   const long long gid0 = static_cast<long long>(blockIdx.x) * C::S + g;
   const long long gstride = static_cast<long long>(gridDim.x) * C::S;
 
+  // Work distribution: the group's first sub-filter is blockIdx.x * S + g;
+  // later ones come from the launch's work counter (dynamic, so SMs that
+  // finish early take more).  Thread 0 announces each next index through
+  // next_s[barrier] before arriving on that barrier (release / acquire), and
+  // a "no more work" index completes the barrier phase without a copy.
+  auto issue = [&](int b, long long nn) {   // thread 0 only
+    next_s[b] = static_cast<unsigned int>(nn < P.n_local ? nn : P.n_local);
+    if (nn < P.n_local) {
+      mbar_arrive_expect_tx(bars + b, static_cast<uint32_t>(C::stage_bytes));
+      bulk_g2s(gs + C::g_stage + b * C::stage_bytes, P.parts + nn * C::ROW, static_cast<uint32_t>(C::stage_bytes),
+               bars + b);
+    } else {
+      mbar_arrive(bars + b);
+    }
+  };
+  auto fetch_next = [&]() -> long long { return gstride + atomicAdd(P.work, 1u); };
+
   if (G.t == 0) {
     mbar_init(bars, 1);
     mbar_init(bars + 1, 1);
     fence_mbar_init();
-    if (gid0 < P.n_local) {
-      mbar_arrive_expect_tx(bars, static_cast<uint32_t>(C::stage_bytes));
-      bulk_g2s(gs + C::g_stage, P.parts + gid0 * C::ROW, static_cast<uint32_t>(C::stage_bytes), bars);
-    }
+    issue(0, gid0);
   }
   if (do_sample) {
     if (threadIdx.x < NJ + 2) z_s[threadIdx.x] = P.z[threadIdx.x];
@@ -480,24 +498,26 @@ __global__ void __launch_bounds__(C::T* C::S) pf_step_kernel(const __grid_consta
   }
   __syncthreads();
 
-  int it = 0;
-  for (long long n = gid0; n < P.n_local; n += gstride, ++it) {
+  for (int it = 0;; ++it) {
     const int st = (C::NSTAGE == 2) ? (it & 1) : 0;
+    mbar_wait(bars + st, C::NSTAGE == 2 ? (it >> 1) & 1 : it & 1);
+    const long long n = next_s[st];
+    if (n >= P.n_local) break;
+    if constexpr (C::NSTAGE == 2) {   // prefetch the next sub-filter into the other stage
+      if (G.t == 0) issue(st ^ 1, fetch_next());
+    }
     float* xs = reinterpret_cast<float*>(gs + C::g_stage + st * C::stage_bytes);
     float* ws = xs + D * M;
     const long long gsf = P.g0 + n;                    // global sub-filter
     const uint32_t pbase = static_cast<uint32_t>(gsf * M);
     float* gblk = P.parts + n * C::ROW;                // this sub-filter's block in HBM
-    if constexpr (C::NSTAGE == 2) {   // prefetch the next sub-filter into the other stage
-      if (G.t == 0 && n + gstride < P.n_local) {
-        mbar_arrive_expect_tx(bars + (st ^ 1), static_cast<uint32_t>(C::stage_bytes));
-        bulk_g2s(gs + C::g_stage + (st ^ 1) * C::stage_bytes, P.parts + (n + gstride) * C::ROW,
-                 static_cast<uint32_t>(C::stage_bytes), bars + (st ^ 1));
+    auto finish = [&]() {   // end of a sub-filter: free the stage, start the next load (NSTAGE 1)
+      fence_proxy_async_smem();
+      gsync<GW>(g);
+      if constexpr (C::NSTAGE == 1) {
+        if (G.t == 0) issue(0, fetch_next());
       }
-      mbar_wait(bars + st, (it >> 1) & 1);
-    } else {
-      mbar_wait(bars, it & 1);
-    }
+    };
 
     float lw[PP];
 #pragma unroll
@@ -617,14 +637,7 @@ __global__ void __launch_bounds__(C::T* C::S) pf_step_kernel(const __grid_consta
     }
 
     if (mode == MODE_EXCHANGE) {
-      fence_proxy_async_smem();
-      gsync<GW>(g);
-      if constexpr (C::NSTAGE == 1) {
-        if (G.t == 0 && n + gstride < P.n_local) {
-          mbar_arrive_expect_tx(bars, static_cast<uint32_t>(C::stage_bytes));
-          bulk_g2s(gs + C::g_stage, P.parts + (n + gstride) * C::ROW, static_cast<uint32_t>(C::stage_bytes), bars);
-        }
-      }
+      finish();
       continue;
     }
 
@@ -653,7 +666,7 @@ __global__ void __launch_bounds__(C::T* C::S) pf_step_kernel(const __grid_consta
           for (int j = 0; j < PP; ++j) mo = max(mo, ord_f32(lw[j]));
           mo = __reduce_max_sync(0xFFFFFFFFu, mo);
           if constexpr (GW > 1) {
-            uint32_t* r = reinterpret_cast<uint32_t*>(G.red + G.rb * 64);
+            uint32_t* r = reinterpret_cast<uint32_t*>(G.red + G.rb * 32);
             G.rb ^= 1;
             if (G.lane == 0) r[G.wig] = mo;
             gsync<GW>(g);
@@ -671,12 +684,14 @@ __global__ void __launch_bounds__(C::T* C::S) pf_step_kernel(const __grid_consta
         for (int j = 0; j < PP; ++j) P.dbg_anc[n * M + C::slot(G.t, j)] = anc[j];
       }
       if constexpr (C::STAGED) {
+        // rolled sample loop: per-slot ancestor -> the (now free) log-weight
+        // row, Philox words -> the (now free) scan buffer; own slots only
+        gsync<GW>(g);
 #pragma unroll
         for (int j = 0; j < PP; ++j) {
           const int s = C::slot(G.t, j);
-          anc_s[s] = anc[j];
-          bz_s[s] = bz[j];
-          bw_s[s] = bw[j];
+          reinterpret_cast<int*>(ws)[s] = anc[j];
+          bzw_s[s] = make_uint2(bz[j], bw[j]);
         }
       }
     }
@@ -691,9 +706,10 @@ __global__ void __launch_bounds__(C::T* C::S) pf_step_kernel(const __grid_consta
         int a;
         uint32_t z2, z3;
         if constexpr (C::STAGED) {
-          a = anc_s[s];
-          z2 = bz_s[s];
-          z3 = bw_s[s];
+          a = reinterpret_cast<const int*>(ws)[s];
+          const uint2 bb = bzw_s[s];
+          z2 = bb.x;
+          z3 = bb.y;
         } else {
           a = anc[j];
           z2 = bz[j];
@@ -748,14 +764,7 @@ __global__ void __launch_bounds__(C::T* C::S) pf_step_kernel(const __grid_consta
         }
       }
     }
-    fence_proxy_async_smem();
-    gsync<GW>(g);
-    if constexpr (C::NSTAGE == 1) {
-      if (G.t == 0 && n + gstride < P.n_local) {
-        mbar_arrive_expect_tx(bars, static_cast<uint32_t>(C::stage_bytes));
-        bulk_g2s(gs + C::g_stage, P.parts + (n + gstride) * C::ROW, static_cast<uint32_t>(C::stage_bytes), bars);
-      }
-    }
+    finish();
   }
 
   // ---- a5: the last CTA to finish copies the winning particle (R6)
@@ -799,6 +808,7 @@ __global__ void __launch_bounds__(C::T* C::S) pf_step_kernel(const __grid_consta
     if (tid == 0) {
       *P.key_next = 0ull;
       *P.counter = 0u;
+      *P.work = 0u;
     }
   }
 }

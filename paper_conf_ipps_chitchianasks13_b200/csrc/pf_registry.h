@@ -16,7 +16,7 @@ struct StepParams;
 
 struct KernelEntry {
   int nj, m, res;
-  int gw, s, nstage, unr;   // warps per sub-filter group, groups per CTA, TMA stages, sample unroll
+  int gw, s, nstage, unr, minb;   // warps per group, groups per CTA, TMA stages, sample unroll, min CTAs/SM
   cudaError_t (*prepare)(int* blocks_per_sm);
   cudaError_t (*launch)(const StepParams& p, int grid, cudaStream_t s);
   cudaError_t (*resample_debug)(const uint32_t* q, const uint32_t* ua, const uint32_t* ub, int* anc,
@@ -32,7 +32,7 @@ extern const KernelEntry kEntriesNJ28[];
 extern const int kNumEntriesNJ28;
 }  // namespace pf
 
-#define PF_ENTRY(NJ, M, RES, GW, S, NST, UNR)                                                             \
+#define PF_ENTRY(NJ, M, RES, GW, S, NST, UNR, MINB)                                                             \
   {NJ,                                                                                                    \
    M,                                                                                                     \
    RES,                                                                                                   \
@@ -40,13 +40,14 @@ extern const int kNumEntriesNJ28;
    S,                                                                                                     \
    NST,                                                                                                   \
    UNR,                                                                                                   \
-   &StepKernel<KCfg<NJ, M, RES, GW, S, NST, UNR>>::prepare,                                               \
-   &StepKernel<KCfg<NJ, M, RES, GW, S, NST, UNR>>::launch,                                                \
-   &StepKernel<KCfg<NJ, M, RES, GW, S, NST, UNR>>::resample_debug,                                        \
-   StepKernel<KCfg<NJ, M, RES, GW, S, NST, UNR>>::smem()}
+   MINB,                                                                                                  \
+   &StepKernel<KCfg<NJ, M, RES, GW, S, NST, UNR, MINB>>::prepare,                                               \
+   &StepKernel<KCfg<NJ, M, RES, GW, S, NST, UNR, MINB>>::launch,                                                \
+   &StepKernel<KCfg<NJ, M, RES, GW, S, NST, UNR, MINB>>::resample_debug,                                        \
+   StepKernel<KCfg<NJ, M, RES, GW, S, NST, UNR, MINB>>::smem()}
 // Default mapping for small states (d <= 12): two particles per thread
 // (rolled per-particle loop), several sub-filters per CTA for small m.
-#define PF_SMALL_D_ENTRIES(NJ, RES)                                                                       \
-  PF_ENTRY(NJ, 32, RES, 1, 8, 2, 1), PF_ENTRY(NJ, 64, RES, 1, 8, 2, 1), PF_ENTRY(NJ, 128, RES, 2, 4, 2, 1), \
-      PF_ENTRY(NJ, 256, RES, 4, 2, 2, 1), PF_ENTRY(NJ, 512, RES, 8, 1, 2, 1),                              \
-      PF_ENTRY(NJ, 1024, RES, 16, 1, 1, 1)
+#define PF_SMALL_D_ENTRIES(NJ, RES)                                                                  \
+  PF_ENTRY(NJ, 32, RES, 1, 8, 2, 1, 1), PF_ENTRY(NJ, 64, RES, 1, 8, 2, 1, 1),                         \
+      PF_ENTRY(NJ, 128, RES, 2, 4, 1, 1, 1), PF_ENTRY(NJ, 256, RES, 4, 2, 2, 1, 1),                   \
+      PF_ENTRY(NJ, 512, RES, 8, 1, 2, 1, 1), PF_ENTRY(NJ, 1024, RES, 16, 1, 1, 1, 1)

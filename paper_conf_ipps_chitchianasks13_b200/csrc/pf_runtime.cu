@@ -24,7 +24,8 @@ constexpr int kStageSlots = 8;
 
 // scratch layout (bytes)
 constexpr size_t kOffKeys = 0;        // u64[2]
-constexpr size_t kOffCounter = 16;    // u32
+constexpr size_t kOffCounter = 16;    // u32 CTA completion counter
+constexpr size_t kOffWork = 20;       // u32 dynamic work counter
 constexpr size_t kOffRecord = 64;     // float[4 + d]  (d <= 32 -> 144 B)
 constexpr size_t kOffInputs = 256;    // float[64]: z at 0, u at 32
 constexpr size_t kOffMu0 = 512;       // float[64]
@@ -166,6 +167,7 @@ pf::StepParams base_params(pf_handle* h, long long k, int mode) {
   p.key_cur = keys(h) + (k & 1);
   p.key_next = keys(h) + ((k + 1) & 1);
   p.counter = reinterpret_cast<unsigned int*>(h->scratch + kOffCounter);
+  p.work = reinterpret_cast<unsigned int*>(h->scratch + kOffWork);
   p.record = record(h);
   p.est_out = nullptr;
   p.dbg_src = nullptr;
