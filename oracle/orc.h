@@ -135,6 +135,14 @@ int orc_s_set(orc_s_filter* f, const float* state, const float* logw, int64_t st
 int orc_s_trace(const orc_s_filter* f, int64_t* src, int32_t* ancestors);
 void orc_s_destroy(orc_s_filter* f);
 
+/* One step k >= 2 for the listed sub-filters only, from the full weighted
+ * set of step k-1 (state [d][M], logw [M]) — exchange, normalise, resample,
+ * sample, weight, one sub-filter at a time.  out_state [d][n_sub*m],
+ * out_logw [n_sub*m].  For sampled checks at full size. */
+int orc_s_step_subset(const orc_config* cfg, const orc_model* md, const float* state, const float* logw,
+                      int64_t k, const float* z, const float* u, const int64_t* subs, int64_t n_sub,
+                      float* out_state, float* out_logw);
+
 orc_d_filter* orc_d_create(const orc_config* cfg, const orc_model* md, const double* mu0,
                            const double* sigma0);
 int orc_d_step(orc_d_filter* f, const double* z, const double* u);

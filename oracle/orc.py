@@ -87,6 +87,7 @@ def lib():
             "orc_s_set": (C.c_int, [P, P, P, C.c_int64]),
             "orc_s_trace": (C.c_int, [P, P, P]),
             "orc_s_destroy": (None, [P]),
+            "orc_s_step_subset": (C.c_int, [P, P, P, P, C.c_int64, P, P, P, C.c_int64, P, P]),
             "orc_d_create": (P, [P, P, P, P]),
             "orc_d_step": (C.c_int, [P, P, P]),
             "orc_d_estimate": (C.c_int, [P, P, P, P]),
@@ -300,6 +301,22 @@ def exchange(cfg: Config, logw) -> np.ndarray:
     if rc:
         raise ValueError(f"orc_s_exchange failed: {rc}")
     return src
+
+
+def step_subset(cfg: Config, model: Model, state, logw, k: int, z, u, subs):
+    """Step k of the listed sub-filters from the full weighted set of step k-1:
+    returns (state [d][len(subs)*m], logw [len(subs)*m])."""
+    st, lw = _f32(state), _f32(logw)
+    sb = np.ascontiguousarray(subs, np.int64)
+    d, m = model.d, cfg.m
+    out_s = np.zeros((d, len(sb) * m), np.float32)
+    out_w = np.zeros(len(sb) * m, np.float32)
+    cc, mc = cfg.c(), model.c()
+    rc = lib().orc_s_step_subset(C.byref(cc), C.byref(mc), _p(st), _p(lw), k, _p(_f32(z)), _p(_f32(u)), _p(sb),
+                                 len(sb), _p(out_s), _p(out_w))
+    if rc:
+        raise ValueError(f"orc_s_step_subset failed: {rc}")
+    return out_s, out_w
 
 
 # ---- the filter -------------------------------------------------------------

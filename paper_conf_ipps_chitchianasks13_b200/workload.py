@@ -70,8 +70,10 @@ def make_trajectory(n_joints: int, T: int, seed: int = 0, h_s: float = 0.1, nois
 def random_particles(traj: dict, M: int, seed: int, spread: float = 0.2):
     """SoA particle set [d][M] scattered around the true state X[1] (float32)."""
     rng = np.random.default_rng(20000 + seed)
-    x = traj["X"][1][:, None] + spread * rng.standard_normal((traj["d"], M))
-    return np.ascontiguousarray(x, np.float32)
+    x = rng.standard_normal((traj["d"], M), dtype=np.float32)   # float32 throughout: 16M x 32 fits
+    x *= np.float32(spread)
+    x += traj["X"][1][:, None].astype(np.float32)
+    return x
 
 
 def random_logw(N: int, m: int, seed: int, ties: bool = True, scale: float = 30.0) -> np.ndarray:

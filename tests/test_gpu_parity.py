@@ -218,3 +218,36 @@ def test_sharded_loopback_bit_identical(P, orc, W, topo, N, world):
     so, wo, _ = o.get()
     sg = np.concatenate([s.get_particles()[0] for s in shards], axis=1)
     np.testing.assert_array_equal(sg, so)
+
+
+@pytest.mark.parametrize("name,nj,m,N,t,topo,res", [
+    ("C4 high-DOF arm 16M, Vose", 28, 256, 65536, 1, "ring", "vose"),
+    ("C5 per-GPU shard 16M, RWS", 5, 256, 65536, 1, "ring", "rws"),
+    ("C3 m=32 at 4M, torus t=4", 5, 32, 131072, 4, "torus", "rws"),
+    ("C3 m=1024 at 4M, torus t=2", 5, 1024, 4096, 2, "torus", "vose"),
+])
+def test_full_size_sampled(P, orc, W, name, nj, m, N, t, topo, res):
+    # BASELINE configs at full size in the bench's launch configuration: one
+    # step from a generator-made weighted set; the oracle recomputes a sample
+    # of sub-filters one by one (exchange, resample, sample, weight)
+    tr = W.make_trajectory(nj, 10, 2)
+    g = P.ParticleFilter(tr["mu0"], tr["sigma0"], P.ArmModel(n_joints=nj), m=m, n_filters=N, t=t, topo=topo,
+                         resampler=res, seed=31337)
+    s0 = W.random_particles(tr, m * N, 5)
+    w0 = W.random_logw(N, m, 5).ravel()
+    g.set_particles(s0, w0, 4)
+    g.step(tr["Z"][5], tr["U"][4])
+    sg, wg, k = g.get_particles()
+    assert k == 5
+    rng = np.random.default_rng(N + m)
+    subs = np.unique(np.concatenate([[0, N - 1, N // 2], rng.integers(0, N, 21)]))
+    cfg = orc.Config(m=m, n_filters=N, t=t, topo=topo, resampler=res, seed=31337)
+    so, wo = orc.step_subset(cfg, orc.Model(n_joints=nj), s0, w0, 5, tr["Z"][5], tr["U"][4], subs)
+    for i, n in enumerate(subs):
+        np.testing.assert_array_equal(sg[:, n * m:(n + 1) * m], so[:, i * m:(i + 1) * m], err_msg=f"{name} sf {n}")
+        np.testing.assert_array_equal(wg[n * m:(n + 1) * m], wo[i * m:(i + 1) * m], err_msg=f"{name} sf {n}")
+    # the estimate is the global argmax of the new log-weights (R6)
+    x, lw, idx = g.estimate()
+    assert lw == wg.max() and idx == int(np.flatnonzero(wg == wg.max())[0])
+    np.testing.assert_array_equal(x, sg[:, idx])
+    g.close()

@@ -113,3 +113,23 @@ def test_fp32_matches_fp64_accuracy(orc, W):
     diff = np.array(r32) - np.array(r64)
     se = np.std(r32 + r64) / np.sqrt(len(r32))
     assert abs(np.mean(diff)) < 3 * se + 1e-3
+
+
+def test_step_subset_equals_whole_filter(orc, W):
+    # the one-sub-filter-at-a-time oracle used for full-size sampled checks
+    # reproduces the whole-filter step exactly
+    for topo, res, t in [("ring", "rws", 1), ("torus", "vose", 2), ("none", "rws", 0)]:
+        cfg = orc.Config(m=32, n_filters=16, t=t, topo=topo, resampler=res, seed=5)
+        md = orc.Model(n_joints=5)
+        tr = W.make_trajectory(5, 10, 0)
+        f = orc.Filter(cfg, md, tr["mu0"], tr["sigma0"])
+        s0 = W.random_particles(tr, 512, 1)
+        w0 = W.random_logw(16, 32, 1).ravel()
+        f.set(s0, w0, 3)
+        f.step(tr["Z"][4], tr["U"][3])
+        s1, w1, _ = f.get()
+        subs = [0, 5, 15, 7]
+        os_, ow = orc.step_subset(cfg, md, s0, w0, 4, tr["Z"][4], tr["U"][3], subs)
+        for i, n in enumerate(subs):
+            np.testing.assert_array_equal(os_[:, i * 32:(i + 1) * 32], s1[:, n * 32:(n + 1) * 32])
+            np.testing.assert_array_equal(ow[i * 32:(i + 1) * 32], w1[n * 32:(n + 1) * 32])
