@@ -132,8 +132,8 @@ struct KCfg {
   static constexpr size_t g_lists = g_alias + (RES == RES_VOSE ? sizeof(int) * M : 0);
   static constexpr size_t g_red = g_lists + (RES == RES_VOSE ? sizeof(int) * M : 0);   // u64 [2][32]
   static constexpr size_t g_cand = g_red + sizeof(u64) * 64;                     // u64 [GW][KMAX+1]
-  static constexpr size_t g_misc = g_cand + sizeof(u64) * GW * (KMAX + 1);       // int [GW][KMAX]
-  static constexpr size_t g_bar = g_misc + sizeof(int) * GW * KMAX;              // u64 [2] + next [2]
+  static constexpr size_t g_misc = g_cand + sizeof(u64) * GW * (KMAX + 1);       // int [GW][2][KMAX]
+  static constexpr size_t g_bar = g_misc + sizeof(int) * GW * 2 * KMAX;          // u64 [2] + next [2]
   static constexpr size_t group_bytes = (g_bar + 32 + 127) / 128 * 128;
   // per-CTA
   static constexpr size_t c_zin = 0;          // float [64]: z (NJ+2), h_s u (NJ)
@@ -317,24 +317,33 @@ __device__ __forceinline__ void resample_group(const uint32_t (&q)[C::P], const 
     // Vose's alias method (PAPER.md:18 §IV, :20–22 §VI-F), table by the
     // closed form of the sequential sweep (R10): a_j = M q_j, small L =
     // {a < Q}, D = inclusive deficits over L, E = inclusive excesses over H.
-    u64 val[P], tmp[P];
+    // Two slot-order scans: the weights (-> Q and the prefix of a = M q), and
+    // the deficits over L with the count of L packed above bit 48 (D < 2^42).
+    // E follows from sum_{j'<=j} (a_j' - Q) = E_j - D_j.
+    u64 val[P], qinc[P];
 #pragma unroll
     for (int j = 0; j < P; ++j) val[j] = q[j];
-    const u64 Q = slot_scan_incl<C, u64>(val, tmp, G);
+    const u64 Q = slot_scan_incl<C, u64>(val, qinc, G);
     u64 a[P];
     bool small[P];
-    u64 cnt_in[P], cnt[P], def[P], Dinc[P], exc[P], Einc[P];
+    u64 packed[P], pinc[P], cnt[P], def[P], Dinc[P], Einc[P];
 #pragma unroll
     for (int j = 0; j < P; ++j) {
       a[j] = static_cast<u64>(M) * q[j];
       small[j] = a[j] < Q;
-      cnt_in[j] = small[j] ? 1ull : 0ull;
       def[j] = small[j] ? Q - a[j] : 0ull;
-      exc[j] = small[j] ? 0ull : a[j] - Q;
+      packed[j] = def[j] + (small[j] ? (1ull << 48) : 0ull);
     }
-    const int nL = static_cast<int>(slot_scan_incl<C, u64>(cnt_in, cnt, G));
-    const u64 Dtot = slot_scan_incl<C, u64>(def, Dinc, G);
-    slot_scan_incl<C, u64>(exc, Einc, G);
+    const u64 ptot = slot_scan_incl<C, u64>(packed, pinc, G);
+    const int nL = static_cast<int>(ptot >> 48);
+    const u64 Dtot = ptot & ((1ull << 48) - 1);
+#pragma unroll
+    for (int j = 0; j < P; ++j) {
+      cnt[j] = pinc[j] >> 48;
+      Dinc[j] = pinc[j] & ((1ull << 48) - 1);
+      const u64 slot1 = static_cast<u64>(C::slot(G.t, j)) + 1;
+      Einc[j] = Dinc[j] + static_cast<u64>(M) * qinc[j] - slot1 * Q;
+    }
 #pragma unroll
     for (int j = 0; j < P; ++j) {
       const int s = C::slot(G.t, j);
@@ -382,23 +391,29 @@ __device__ __forceinline__ void resample_group(const uint32_t (&q)[C::P], const 
 }
 
 // ------------------------------------------------------------ topology
-__device__ __forceinline__ long long neighbor_of(const StepParams& P, long long g, int qi) {
-  if (P.topo == TOPO_RING) return qi == 0 ? (g - 1 + P.n_global) % P.n_global : (g + 1) % P.n_global;
-  const long long r = g / P.C, c = g % P.C;
-  switch (qi) {
-    case 0: return ((r - 1 + P.R) % P.R) * P.C + c;
-    case 1: return ((r + 1) % P.R) * P.C + c;
-    case 2: return r * P.C + (c - 1 + P.C) % P.C;
-    default: return r * P.C + (c + 1) % P.C;
+// Mailbox row of neighbour qi of local sub-filter g (global index) — rows
+// [0, n_local) are the shard's own sub-filters, [n_local, n_ext) the halo
+// rows of pf.h pf_shard.  Ring (R3): [g-1, g+1] mod N; 2D torus (R4): [up,
+// down, left, right] with wrap; a shard holds whole grid rows, so left/right
+// are always local and up/down leave the shard only at its first/last row.
+__device__ __forceinline__ long long neighbor_row(const StepParams& P, long long g, int qi) {
+  const long long N = P.n_global;
+  if (P.topo == TOPO_RING) {
+    const long long q = qi == 0 ? (g == 0 ? N - 1 : g - 1) : (g == N - 1 ? 0 : g + 1);
+    const long long loc = q - P.g0;
+    if (loc >= 0 && loc < P.n_local) return loc;
+    return qi == 0 ? P.n_local : P.n_local + 1;
   }
-}
-// mailbox row of global sub-filter q: local rows, then halo rows (pf.h pf_shard)
-__device__ __forceinline__ long long mailbox_row(const StepParams& P, long long q) {
-  const long long loc = q - P.g0;
-  if (loc >= 0 && loc < P.n_local) return loc;
-  if (P.topo == TOPO_RING) return q == (P.g0 - 1 + P.n_global) % P.n_global ? P.n_local : P.n_local + 1;
-  const long long rq = q / P.C, cq = q % P.C, r0 = P.g0 / P.C;
-  return rq == (r0 - 1 + P.R) % P.R ? P.n_local + cq : P.n_local + P.C + cq;
+  const int C = static_cast<int>(P.C), R = static_cast<int>(P.R);
+  const int loc = static_cast<int>(g - P.g0);
+  const int lr = loc / C, c = loc - lr * C;
+  const int rows = static_cast<int>(P.n_local / C);
+  switch (qi) {
+    case 0: return lr > 0 ? loc - C : (rows == R ? (R - 1) * C + c : static_cast<int>(P.n_local) + c);
+    case 1: return lr < rows - 1 ? loc + C : (rows == R ? c : static_cast<int>(P.n_local) + C + c);
+    case 2: return lr * C + (c == 0 ? C - 1 : c - 1);
+    default: return lr * C + (c == C - 1 ? 0 : c + 1);
+  }
 }
 
 // ------------------------------------------------------------ sampling
@@ -459,7 +474,8 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
   G.red = reinterpret_cast<u64*>(gs + C::g_red);
   G.rb = 0;
   u64* cand = reinterpret_cast<u64*>(gs + C::g_cand);             // [GW][KMAX+1]
-  int* wlist = reinterpret_cast<int*>(gs + C::g_misc) + G.wig * C::KMAX;   // this warp's copy
+  int* wlist = reinterpret_cast<int*>(gs + C::g_misc) + G.wig * 2 * C::KMAX;   // this warp's copy: worst slots
+  int* woff = wlist + C::KMAX;                                                  // mailbox offsets of the incoming
 
   const int mode = P.mode;
   const bool do_merge = (mode == MODE_EXCHANGE) || (mode == MODE_STEP && !P.first);
@@ -529,25 +545,29 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
     if (do_merge && K > 0) {
       // worst K by order key (ascending = worse, R6): per-warp bottom-K by
       // K rounds of warp REDUX, then a merge of the GW lists after one barrier
-      uint32_t excl = 0;
+      u64 key[PP];
       uint32_t wmax = 0;
 #pragma unroll
-      for (int j = 0; j < PP; ++j) wmax = max(wmax, ord_f32(lw[j]));
+      for (int i = 0; i < PP; ++i) {
+        key[i] = order_key(lw[i], static_cast<uint32_t>(C::slot(G.t, i)));
+        wmax = max(wmax, static_cast<uint32_t>(key[i] >> 32));
+      }
       wmax = __reduce_max_sync(0xFFFFFFFFu, wmax);
+      // incoming item j = (neighbour j / t, its j % t-th best): mailbox offset
+      if (G.lane < K) {
+        const int qi = G.lane / P.t;
+        woff[G.lane] = static_cast<int>((neighbor_row(P, gsf, qi) * P.tt + (G.lane - qi * P.t)) * E);
+      }
       u64 my_cand = ~0ull;
 #pragma unroll 1
       for (int j = 0; j < K; ++j) {
-        u64 mk = ~0ull;
+        u64 mk = key[0];
 #pragma unroll
-        for (int i = 0; i < PP; ++i) {
-          const u64 key = (excl >> i) & 1u ? ~0ull : order_key(lw[i], static_cast<uint32_t>(C::slot(G.t, i)));
-          mk = key < mk ? key : mk;
-        }
+        for (int i = 1; i < PP; ++i) mk = key[i] < mk ? key[i] : mk;
         const u64 wk = warp_min_u64(mk);
-        const int slot = static_cast<int>(0xFFFFFFFFu - static_cast<uint32_t>(wk));
 #pragma unroll
         for (int i = 0; i < PP; ++i)
-          if (C::slot(G.t, i) == slot) excl |= 1u << i;
+          if (key[i] == wk) key[i] = ~0ull;   // keys are unique (slot in the low bits)
         if (G.lane == j) my_cand = wk;
       }
       if constexpr (GW == 1) {
@@ -582,24 +602,19 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
           if (G.lane == j) mine = wk;
         }
         if (G.lane < K) wlist[G.lane] = static_cast<int>(0xFFFFFFFFu - static_cast<uint32_t>(mine));
-        // own slots among the final worst K
-        excl = 0;
-        __syncwarp();
-#pragma unroll 1
-        for (int j = 0; j < K; ++j) {
-          const int s = wlist[j];
-#pragma unroll
-          for (int i = 0; i < PP; ++i)
-            if (C::slot(G.t, i) == s) excl |= 1u << i;
-        }
       }
       __syncwarp();
+      // own slots among the worst K (slot s is owned by thread s mod T, index s / T)
+      uint32_t excl = 0;
+#pragma unroll 1
+      for (int j = 0; j < K; ++j) {
+        const int s = wlist[j];
+        if ((s & (C::T - 1)) == G.t) excl |= 1u << (s / C::T);
+      }
 #pragma unroll 1
       for (int e = G.t; e < K * E; e += C::T) {
         const int j = e / E, c = e - j * E;
-        const int qi = j / P.t, jj = j - qi * P.t;
-        const long long row = mailbox_row(P, neighbor_of(P, gsf, qi));
-        const float v = P.mb_prev[(row * P.tt + jj) * E + c];
+        const float v = P.mb_prev[woff[j] + c];
         const int slot = wlist[j];
         if (c == 0) ws[slot] = v;
         else if (c >= 2) xs[(c - 2) * M + slot] = v;
@@ -612,11 +627,7 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
           if ((excl >> i) & 1u)
 #pragma unroll 1
             for (int j = 0; j < K; ++j)
-              if (wlist[j] == s) {
-                const int qi = j / P.t, jj = j - qi * P.t;
-                const long long row = mailbox_row(P, neighbor_of(P, gsf, qi));
-                src = __float_as_uint(P.mb_prev[(row * P.tt + jj) * E + 1]);
-              }
+              if (wlist[j] == s) src = __float_as_uint(P.mb_prev[woff[j] + 1]);
           P.dbg_src[n * M + s] = src;
         }
       }

@@ -45,9 +45,10 @@ extern const int kNumEntriesNJ28;
    &StepKernel<KCfg<NJ, M, RES, GW, S, NST, UNR, MINB>>::launch,                                                \
    &StepKernel<KCfg<NJ, M, RES, GW, S, NST, UNR, MINB>>::resample_debug,                                        \
    StepKernel<KCfg<NJ, M, RES, GW, S, NST, UNR, MINB>>::smem()}
-// Default mapping for small states (d <= 12): two particles per thread
-// (rolled per-particle loop), several sub-filters per CTA for small m.
+// Default mapping for small states (d <= 12), measured on B200:
+// about four particles per thread (P = m / 32 GW), one warp per sub-filter up
+// to m = 128, several sub-filters per CTA, at most ~80 registers (3 CTAs/SM).
 #define PF_SMALL_D_ENTRIES(NJ, RES)                                                                  \
-  PF_ENTRY(NJ, 32, RES, 1, 8, 2, 1, 1), PF_ENTRY(NJ, 64, RES, 1, 8, 2, 1, 1),                         \
-      PF_ENTRY(NJ, 128, RES, 2, 4, 1, 1, 1), PF_ENTRY(NJ, 256, RES, 4, 2, 2, 1, 1),                   \
-      PF_ENTRY(NJ, 512, RES, 8, 1, 2, 1, 1), PF_ENTRY(NJ, 1024, RES, 16, 1, 1, 1, 1)
+  PF_ENTRY(NJ, 32, RES, 1, 8, 1, 1, 3), PF_ENTRY(NJ, 64, RES, 1, 8, 1, 1, 3),                       \
+      PF_ENTRY(NJ, 128, RES, 1, 8, 1, 1, 3), PF_ENTRY(NJ, 256, RES, 2, 4, 1, 1, 3),                 \
+      PF_ENTRY(NJ, 512, RES, 4, 2, 1, 1, 3), PF_ENTRY(NJ, 1024, RES, 4, 1, 1, 1, 3)

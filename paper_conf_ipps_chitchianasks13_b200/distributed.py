@@ -13,7 +13,7 @@ of grid rows (2D torus).  The only cross-rank data per step are
 Both go through ``torch.distributed`` (NCCL on GPUs, gloo in the CPU tests).
 The halo *plan* (which mailbox rows go where) is a pure function shared by the
 NCCL path, the single-process loopback used on one GPU, and the gloo tests;
-the kernel side of the same layout is ``mailbox_row`` in csrc/pf_kernels.cuh
+the kernel side of the same layout is ``neighbor_row`` in csrc/pf_kernels.cuh
 and the pf_shard comment in include/pf.h.
 """
 from __future__ import annotations
