@@ -142,8 +142,10 @@ pf_status pf_init(const pf_config* cfg, const pf_model_params* model, const pf_b
  * with the neighbours' best t of step k-1 (l.10–14), normalise + resample
  * locally (l.15–19), sample + weight (l.3–6), local/global estimate (l.8–9).
  * z_k: float[n_joints + 2] = (x_C, y_C, theta_hat_0..), u_{k-1}:
- * float[n_joints].  Host pointers (copied to the device
- * inside the call's stream work) unless PF_DEVICE_INPUTS.  Asynchronous.
+ * float[n_joints].  Host pointers — their values travel to
+ * the device inside the kernel launch, so the buffers may be reused as soon
+ * as the call returns — unless PF_DEVICE_INPUTS (device pointers, read by the
+ * kernel).  Asynchronous.
  * With world > 1 the caller must have filled the halo rows of mailbox
  * parity (k-1)&1 (see pf_shard) and, after the step, reduce the per-rank
  * records (pf_reduce_records) for a global estimate. */

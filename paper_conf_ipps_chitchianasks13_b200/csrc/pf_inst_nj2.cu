@@ -3,6 +3,7 @@
 #include "pf_registry.h"
 
 namespace pf {
-const KernelEntry kEntriesNJ2[] = {PF_SMALL_D_ENTRIES(2, 0), PF_SMALL_D_ENTRIES(2, 1)};
+const KernelEntry kEntriesNJ2[] = {PF_SMALL_D_ENTRIES(2, 0), PF_SMALL_D_ENTRIES(2, 1),
+    PF_LATENCY_ENTRIES(2, 0), PF_LATENCY_ENTRIES(2, 1)};
 const int kNumEntriesNJ2 = sizeof(kEntriesNJ2) / sizeof(kEntriesNJ2[0]);
 }  // namespace pf

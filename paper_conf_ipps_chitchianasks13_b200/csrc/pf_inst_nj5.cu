@@ -7,6 +7,7 @@
 namespace pf {
 const KernelEntry kEntriesNJ5[] = {
     PF_SMALL_D_ENTRIES(5, 0), PF_SMALL_D_ENTRIES(5, 1),
+    PF_LATENCY_ENTRIES(5, 0), PF_LATENCY_ENTRIES(5, 1),
     // alternatives for PF_VARIANT tuning of configs C2 / C5 (m = 256)
     PF_ENTRY(5, 256, 0, 8, 1, 2, 1, 4), PF_ENTRY(5, 256, 0, 1, 8, 1, 1, 3), PF_ENTRY(5, 256, 0, 4, 2, 1, 1, 3),
     PF_ENTRY(5, 256, 1, 8, 1, 2, 1, 2), PF_ENTRY(5, 256, 1, 4, 2, 1, 1, 2),

@@ -47,14 +47,15 @@ struct StepParams {
   float* parts;            // [n_local][D+1][M] blocked SoA (row D = log-weight)
   const float* mb_prev;    // mailbox parity (k-1)&1 : [n_ext][tt][E]
   float* mb_cur;           // mailbox parity k&1
-  const float* z;          // [NJ+2] device
-  const float* u;          // [NJ]   device
+  const float* z;          // [NJ+2] device, or nullptr: use zin
+  const float* u;          // [NJ]   device, or nullptr: use uin
   u64* key_cur;            // global best key of this step (0 on entry)
   u64* key_next;           // reset to 0 for the next step
   unsigned int* counter;   // CTA completion counter (0 on entry, reset by the last CTA)
   unsigned int* work;      // dynamic sub-filter counter (0 on entry, reset by the last CTA)
   float* record;           // [4 + d] estimate record of this shard
   float* est_out;          // nullable [4 + d] (batched mode)
+  float* record_host;      // nullable [4 + d]: mapped pinned host copy of the record
   long long* dbg_src;      // nullable [M_local] exchange sources (global index)
   int* dbg_anc;            // nullable [M_local] ancestors
   long long n_local, g0, n_global, R, C;
@@ -62,6 +63,8 @@ struct StepParams {
   uint32_t k;
   int mode, first;
   uint32_t rk[20];         // Philox round keys (key0 + r W0, key1 + r W1), r = 0..9
+  float zin[32];           // step inputs carried by the launch itself (host-input mode)
+  float uin[32];
 };
 
 // ------------------------------------------------------------- PTX helpers
@@ -509,8 +512,8 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
     issue(0, gid0);
   }
   if (do_sample) {
-    if (threadIdx.x < NJ + 2) z_s[threadIdx.x] = P.z[threadIdx.x];
-    if (threadIdx.x < NJ) hsu_s[threadIdx.x] = P.mc.hs * P.u[threadIdx.x];
+    if (threadIdx.x < NJ + 2) z_s[threadIdx.x] = P.z ? P.z[threadIdx.x] : P.zin[threadIdx.x];
+    if (threadIdx.x < NJ) hsu_s[threadIdx.x] = P.mc.hs * (P.u ? P.u[threadIdx.x] : P.uin[threadIdx.x]);
   }
   __syncthreads();
 
@@ -795,25 +798,21 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
       const uint32_t gidx = 0xFFFFFFFFu - static_cast<uint32_t>(key);
       const long long col = static_cast<long long>(gidx) - P.g0 * M;
       const float* blk = P.parts + (col / M) * C::ROW + (col % M);
+      float* outs[3] = {P.record, P.est_out, P.record_host};
       if (tid < D) {
         const float v = __ldcg(blk + tid * M);
-        P.record[4 + tid] = v;
-        if (P.est_out) P.est_out[4 + tid] = v;
+#pragma unroll
+        for (int o = 0; o < 3; ++o)
+          if (outs[o]) outs[o][4 + tid] = v;
       }
       if (tid == 0) {
-        const float r0 = __uint_as_float(static_cast<uint32_t>(key));
-        const float r1 = __uint_as_float(static_cast<uint32_t>(key >> 32));
-        const float r2 = unord_f32(static_cast<uint32_t>(key >> 32));
-        P.record[0] = r0;
-        P.record[1] = r1;
-        P.record[2] = r2;
-        P.record[3] = 0.0f;
-        if (P.est_out) {
-          P.est_out[0] = r0;
-          P.est_out[1] = r1;
-          P.est_out[2] = r2;
-          P.est_out[3] = 0.0f;
-        }
+        const float r[4] = {__uint_as_float(static_cast<uint32_t>(key)), __uint_as_float(static_cast<uint32_t>(key >> 32)),
+                            unord_f32(static_cast<uint32_t>(key >> 32)), 0.0f};
+#pragma unroll
+        for (int o = 0; o < 3; ++o)
+          if (outs[o])
+#pragma unroll
+            for (int c = 0; c < 4; ++c) outs[o][c] = r[c];
       }
     }
     if (tid == 0) {

@@ -52,3 +52,8 @@ extern const int kNumEntriesNJ28;
   PF_ENTRY(NJ, 32, RES, 1, 8, 1, 1, 3), PF_ENTRY(NJ, 64, RES, 1, 8, 1, 1, 3),                       \
       PF_ENTRY(NJ, 128, RES, 1, 8, 1, 1, 3), PF_ENTRY(NJ, 256, RES, 2, 4, 1, 1, 3),                 \
       PF_ENTRY(NJ, 512, RES, 4, 2, 1, 1, 3), PF_ENTRY(NJ, 1024, RES, 4, 1, 1, 1, 3)
+// Lowest-latency mappings (one particle per thread) for small problems
+// (selected by the runtime when the default leaves most groups idle).
+#define PF_LATENCY_ENTRIES(NJ, RES)                                                                  \
+  PF_ENTRY(NJ, 64, RES, 2, 4, 1, 1, 3), PF_ENTRY(NJ, 128, RES, 4, 2, 1, 1, 3),                      \
+      PF_ENTRY(NJ, 256, RES, 8, 1, 1, 1, 3)

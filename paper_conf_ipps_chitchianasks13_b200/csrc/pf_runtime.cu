@@ -2,7 +2,7 @@
 //
 // Owns host metadata only: configuration validation, shard geometry, the
 // scratch carve-up of the caller's buffers, the kernel table lookup, the
-// per-step launch parameters, and small pinned staging for step inputs.
+// per-step launch parameters (step inputs travel inside the launch).
 // Every computation of the path runs in the kernels of pf_kernels.cuh.
 #include <cuda_runtime.h>
 
@@ -20,7 +20,6 @@ using pf::u64;
 namespace {
 
 constexpr int kMaxNJ = 28;
-constexpr int kStageSlots = 8;
 
 // scratch layout (bytes)
 constexpr size_t kOffKeys = 0;        // u64[2]
@@ -58,6 +57,21 @@ const pf::KernelEntry* find_entry(int nj, int m, int res) {
       }
   }
   return first;
+}
+
+// Small problems (too few sub-filters to keep the default mapping's groups
+// busy) are latency-bound: take the matching entry with the fewest particles
+// per thread.  PF_VARIANT, when set, wins.
+const pf::KernelEntry* latency_entry(int nj, int m, int res) {
+  const pf::KernelEntry* best = nullptr;
+  for (int ti = 0; ti < 3; ++ti) {
+    const Table t = tables(ti);
+    for (int i = 0; i < t.n; ++i)
+      if (t.e[i].nj == nj && t.e[i].m == m && t.e[i].res == res &&
+          (!best || t.e[i].gw > best->gw))
+        best = &t.e[i];
+  }
+  return best;
 }
 
 struct Geometry {
@@ -131,12 +145,11 @@ struct pf_handle {
   const pf::KernelEntry* ke;
   int grid;
   pf_status err;
-  float* pinned;                 // [kStageSlots][64]
-  cudaEvent_t stage_ev[kStageSlots];
-  int stage_next;
   bool trace;
   long long* d_src;
   int* d_anc;
+  float* rec_host;     // mapped pinned host copy of the estimate record (written by the kernels)
+  float* rec_host_dev; // its device alias
   float* d_reduce_tmp;
 };
 
@@ -162,13 +175,14 @@ pf::StepParams base_params(pf_handle* h, long long k, int mode) {
   p.parts = h->parts;
   p.mb_prev = mailbox_parity(h, k - 1);
   p.mb_cur = mailbox_parity(h, k);
-  p.z = inputs(h);
-  p.u = inputs(h) + 32;
+  p.z = nullptr;   // host-input mode: zin / uin (filled by the caller)
+  p.u = nullptr;
   p.key_cur = keys(h) + (k & 1);
   p.key_next = keys(h) + ((k + 1) & 1);
   p.counter = reinterpret_cast<unsigned int*>(h->scratch + kOffCounter);
   p.work = reinterpret_cast<unsigned int*>(h->scratch + kOffWork);
   p.record = record(h);
+  p.record_host = h->rec_host_dev;
   p.est_out = nullptr;
   p.dbg_src = nullptr;
   p.dbg_anc = nullptr;
@@ -193,18 +207,13 @@ pf::StepParams base_params(pf_handle* h, long long k, int mode) {
   return p;
 }
 
-// Copy z (n_j+2) and u (n_j) host -> device inputs through a pinned slot.
-pf_status stage_inputs(pf_handle* h, const float* z, const float* u) {
-  const int nj = h->g.nj;
-  float* slot = h->pinned + h->stage_next * 64;
-  cudaError_t e = cudaEventSynchronize(h->stage_ev[h->stage_next]);
-  if (e != cudaSuccess) return sticky(h, e);
-  std::memcpy(slot, z, sizeof(float) * (nj + 2));
-  std::memcpy(slot + 32, u, sizeof(float) * nj);
-  e = cudaMemcpyAsync(inputs(h), slot, sizeof(float) * (32 + nj), cudaMemcpyHostToDevice, h->stream);
-  if (e == cudaSuccess) e = cudaEventRecord(h->stage_ev[h->stage_next], h->stream);
-  h->stage_next = (h->stage_next + 1) % kStageSlots;
-  return sticky(h, e);
+// Host step inputs travel inside the launch (StepParams.zin / uin): no
+// separate copy, no staging buffer, nothing to synchronize.
+void host_inputs(pf_handle* h, pf::StepParams& p, const float* z, const float* u) {
+  p.z = nullptr;
+  p.u = nullptr;
+  std::memcpy(p.zin, z, sizeof(float) * (h->g.nj + 2));
+  std::memcpy(p.uin, u, sizeof(float) * h->g.nj);
 }
 
 pf_status launch(pf_handle* h, const pf::StepParams& p) {
@@ -236,7 +245,7 @@ __global__ void pf_init_kernel(float* parts, int m, long long M_local, uint32_t 
 }
 
 // Pick the record with the maximal key among `count` (exact, order-free).
-__global__ void pf_reduce_records_kernel(const float* recs, int count, int rec_floats, float* out) {
+__global__ void pf_reduce_records_kernel(const float* recs, int count, int rec_floats, float* out, float* out_host) {
   const int lane = threadIdx.x;
   u64 best = 0ull;
   int bi = 0;
@@ -255,7 +264,11 @@ __global__ void pf_reduce_records_kernel(const float* recs, int count, int rec_f
   const unsigned mask = __ballot_sync(0xFFFFFFFFu, best == win);
   const int src_lane = __ffs(mask) - 1;
   const int src = __shfl_sync(0xFFFFFFFFu, bi, src_lane);
-  for (int c = lane; c < rec_floats; c += 32) out[c] = recs[src * rec_floats + c];
+  for (int c = lane; c < rec_floats; c += 32) {
+    const float v = recs[src * rec_floats + c];
+    out[c] = v;
+    if (out_host) out_host[c] = v;
+  }
 }
 
 // host [d][M_local] rows <-> device blocked [n_local][d+1][m]: row c of the
@@ -320,15 +333,28 @@ pf_status pf_init(const pf_config* cfg, const pf_model_params* model, const pf_b
   if (e == cudaSuccess) e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
   if (e == cudaSuccess) e = h->ke->prepare(&bps);
   if (e == cudaSuccess && bps < 1) e = cudaErrorInvalidConfiguration;
-  if (e == cudaSuccess) e = cudaMallocHost(reinterpret_cast<void**>(&h->pinned), sizeof(float) * 64 * kStageSlots);
-  for (int i = 0; i < kStageSlots && e == cudaSuccess; ++i)
-    e = cudaEventCreateWithFlags(&h->stage_ev[i], cudaEventDisableTiming);
+  if (e == cudaSuccess)
+    e = cudaHostAlloc(reinterpret_cast<void**>(&h->rec_host), sizeof(float) * 64, cudaHostAllocMapped);
+  if (e == cudaSuccess) e = cudaHostGetDevicePointer(reinterpret_cast<void**>(&h->rec_host_dev), h->rec_host, 0);
   if (e != cudaSuccess) {
     pf_destroy(h);
     return PF_ECUDA;
   }
+  // fewer sub-filters than a quarter of the default mapping's groups: switch
+  // to the lowest-latency mapping (more threads per sub-filter)
+  if (!std::getenv("PF_VARIANT") && g.n_local * 4 <= static_cast<long long>(bps) * sms * h->ke->s) {
+    const pf::KernelEntry* le = latency_entry(g.nj, g.m, cfg->resampler);
+    if (le && le != h->ke) {
+      int b2 = 0;
+      if (le->prepare(&b2) == cudaSuccess && b2 >= 1) {
+        h->ke = le;
+        bps = b2;
+      }
+    }
+  }
+  const long long ctas_needed = (g.n_local + h->ke->s - 1) / h->ke->s;
   const long long grid = static_cast<long long>(bps) * sms;
-  h->grid = static_cast<int>(grid < g.n_local ? grid : g.n_local);
+  h->grid = static_cast<int>(grid < ctas_needed ? grid : ctas_needed);
   // scratch: zero keys / counter; prior parameters
   float prior[128];
   std::memset(prior, 0, sizeof(prior));
@@ -365,8 +391,7 @@ pf_status pf_step(pf_handle* h, const float* z_k, const float* u_km1) {
     p.z = z_k;
     p.u = u_km1;
   } else {
-    const pf_status s = stage_inputs(h, z_k, u_km1);
-    if (s != PF_OK) return s;
+    host_inputs(h, p, z_k, u_km1);
   }
   if (h->trace) {
     p.dbg_src = h->d_src;
@@ -403,10 +428,12 @@ pf_status pf_estimate(pf_handle* h, float* x_hat, float* logw, int64_t* idx) {
   if (!h || !x_hat) return PF_EINVAL;
   if (h->err != PF_OK) return h->err;
   if (h->step < 1) return PF_ESTATE;
-  float rec[4 + 32 + 4];
-  cudaError_t e = cudaMemcpyAsync(rec, record(h), sizeof(float) * (4 + h->g.d), cudaMemcpyDeviceToHost, h->stream);
-  if (e == cudaSuccess) e = cudaStreamSynchronize(h->stream);
+  // the kernels wrote the record into mapped pinned host memory: a stream
+  // synchronization is the whole device -> host transfer
+  cudaError_t e = cudaStreamSynchronize(h->stream);
   if (e != cudaSuccess) return sticky(h, e);
+  float rec[4 + 32 + 4];
+  std::memcpy(rec, const_cast<const float*>(h->rec_host), sizeof(float) * (4 + h->g.d));
   uint32_t lo;
   std::memcpy(&lo, &rec[0], 4);
   std::memcpy(x_hat, rec + 4, sizeof(float) * h->g.d);
@@ -425,7 +452,7 @@ pf_status pf_record_ptr(pf_handle* h, float** record_dev, int32_t* record_floats
 pf_status pf_reduce_records(pf_handle* h, const float* records_dev, int32_t count) {
   if (!h || !records_dev || count < 1) return PF_EINVAL;
   if (h->err != PF_OK) return h->err;
-  pf_reduce_records_kernel<<<1, 32, 0, h->stream>>>(records_dev, count, 4 + h->g.d, record(h));
+  pf_reduce_records_kernel<<<1, 32, 0, h->stream>>>(records_dev, count, 4 + h->g.d, record(h), h->rec_host_dev);
   return sticky(h, cudaGetLastError());
 }
 
@@ -485,10 +512,9 @@ pf_status pf_debug_sample_weight(pf_handle* h, const float* state_in, const floa
     e = rows_to_device(h, state_in, 0, h->g.d);
   if (e == cudaSuccess) e = cudaMemsetAsync(keys(h), 0, 2 * sizeof(u64), h->stream);
   if (e != cudaSuccess) return sticky(h, e);
-  pf_status s = stage_inputs(h, z_k, u_km1);
-  if (s != PF_OK) return s;
   pf::StepParams p = base_params(h, k, pf::MODE_SAMPLE);
-  s = launch(h, p);
+  host_inputs(h, p, z_k, u_km1);
+  pf_status s = launch(h, p);
   if (s != PF_OK) return s;
   h->step = k;
   e = cudaStreamSynchronize(h->stream);
@@ -582,10 +608,8 @@ pf_status pf_get_trace(pf_handle* h, int64_t* src, int32_t* ancestors) {
 
 pf_status pf_destroy(pf_handle* h) {
   if (!h) return PF_OK;
-  if (h->stream || true) cudaStreamSynchronize(h->stream);
-  for (int i = 0; i < kStageSlots; ++i)
-    if (h->stage_ev[i]) cudaEventDestroy(h->stage_ev[i]);
-  if (h->pinned) cudaFreeHost(h->pinned);
+  cudaStreamSynchronize(h->stream);
+  if (h->rec_host) cudaFreeHost(h->rec_host);
   if (h->d_src) cudaFree(h->d_src);
   if (h->d_anc) cudaFree(h->d_anc);
   delete h;
