@@ -110,8 +110,9 @@ __device__ __forceinline__ void mbar_wait(u64* bar, uint32_t parity) {
 // group; the per-particle sample/weight loop over a thread's P slots is
 // unrolled UNR times (P for full unrolling; 1 keeps one copy of the
 // ~10–40 KB per-particle code in the instruction cache).
-template <int NJ_, int M_, int RES_, int GW_, int S_, int NSTAGE_, int UNR_, int MINB_>
+template <int NJ_, int M_, int RES_, int GW_, int S_, int NSTAGE_, int UNR_, int MINB_, int EARLY_ = 0>
 struct KCfg {
+  static constexpr int EARLY = EARLY_;       // start the next TMA load right after the sample loop
   static constexpr int NJ = NJ_, M = M_, RES = RES_, GW = GW_, S = S_, NSTAGE = NSTAGE_, UNR = UNR_;
   static constexpr int MINB = MINB_;         // __launch_bounds__ min CTAs per SM (register cap)
   static constexpr int D = NJ + 4;
@@ -503,13 +504,21 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
       mbar_arrive(bars + b);
     }
   };
-  auto fetch_next = [&]() -> long long { return gstride + atomicAdd(P.work, 1u); };
+  // thread 0 keeps one dynamic index in flight: the atomic's latency is
+  // hidden behind a whole sub-filter of work
+  unsigned int pending = 0;
+  auto fetch_next = [&]() -> long long {
+    const long long nn = gstride + pending;
+    pending = atomicAdd(P.work, 1u);
+    return nn;
+  };
 
   if (G.t == 0) {
     mbar_init(bars, 1);
     mbar_init(bars + 1, 1);
     fence_mbar_init();
     issue(0, gid0);
+    if (gid0 < P.n_local) pending = atomicAdd(P.work, 1u);
   }
   if (do_sample) {
     if (threadIdx.x < NJ + 2) z_s[threadIdx.x] = P.z ? P.z[threadIdx.x] : P.zin[threadIdx.x];
@@ -530,11 +539,20 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
     const long long gsf = P.g0 + n;                    // global sub-filter
     const uint32_t pbase = static_cast<uint32_t>(gsf * M);
     float* gblk = P.parts + n * C::ROW;                // this sub-filter's block in HBM
-    auto finish = [&]() {   // end of a sub-filter: free the stage, start the next load (NSTAGE 1)
+    bool issued = false;   // NSTAGE 1: next load already started (after the sample loop)
+    auto release_stage = [&]() {   // all generic smem accesses to the stage done: start the next load
       fence_proxy_async_smem();
       gsync<GW>(g);
       if constexpr (C::NSTAGE == 1) {
         if (G.t == 0) issue(0, fetch_next());
+      }
+      issued = true;
+    };
+    auto finish = [&]() {   // end of a sub-filter
+      if (!issued) {
+        release_stage();
+      } else {
+        gsync<GW>(g);   // the scan region (new log-weights) is reused by the next sub-filter
       }
     };
 
@@ -697,10 +715,11 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
 #pragma unroll
         for (int j = 0; j < PP; ++j) P.dbg_anc[n * M + C::slot(G.t, j)] = anc[j];
       }
+      // all resampler reads of the scan buffer and the log-weight row are done
+      gsync<GW>(g);
       if constexpr (C::STAGED) {
         // rolled sample loop: per-slot ancestor -> the (now free) log-weight
         // row, Philox words -> the (now free) scan buffer; own slots only
-        gsync<GW>(g);
 #pragma unroll
         for (int j = 0; j < PP; ++j) {
           const int s = C::slot(G.t, j);
@@ -739,15 +758,21 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
 #pragma unroll
         for (int c = 0; c < D; ++c) out[c * M] = xo[c];
         out[D * M] = l;
-        ws[s] = l;   // own slot: read back below by this thread only
+        reinterpret_cast<float*>(bzw_s)[2 * s] = l;   // own slot, after its Philox words were read
+
       }
     }
+
+    // the stage buffer is no longer read (new states live in HBM, new
+    // log-weights in the scan buffer): start the next sub-filter's load now
+    if (C::EARLY && do_sample) release_stage();
 
     // ---- a4 local reduce: best t -> mailbox (k&1); a5 global best key
     {
       float lnew[PP];
 #pragma unroll
-      for (int j = 0; j < PP; ++j) lnew[j] = do_sample ? ws[C::slot(G.t, j)] : lw[j];
+      for (int j = 0; j < PP; ++j)
+        lnew[j] = do_sample ? reinterpret_cast<const float*>(bzw_s)[2 * C::slot(G.t, j)] : lw[j];
       uint32_t done = 0;
       const int nbest = P.t > 0 ? P.t : 1;
 #pragma unroll 1

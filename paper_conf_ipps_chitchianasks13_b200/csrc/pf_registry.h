@@ -57,3 +57,9 @@ extern const int kNumEntriesNJ28;
 #define PF_LATENCY_ENTRIES(NJ, RES)                                                                  \
   PF_ENTRY(NJ, 64, RES, 2, 4, 1, 1, 3), PF_ENTRY(NJ, 128, RES, 4, 2, 1, 1, 3),                      \
       PF_ENTRY(NJ, 256, RES, 8, 1, 1, 1, 3)
+#define PF_ENTRY_E(NJ, M, RES, GW, S, NST, UNR, MINB, EARLY)                                      \
+  {NJ, M, RES, GW, S, NST, UNR, MINB,                                                                \
+   &StepKernel<KCfg<NJ, M, RES, GW, S, NST, UNR, MINB, EARLY>>::prepare,                             \
+   &StepKernel<KCfg<NJ, M, RES, GW, S, NST, UNR, MINB, EARLY>>::launch,                              \
+   &StepKernel<KCfg<NJ, M, RES, GW, S, NST, UNR, MINB, EARLY>>::resample_debug,                      \
+   StepKernel<KCfg<NJ, M, RES, GW, S, NST, UNR, MINB, EARLY>>::smem()}

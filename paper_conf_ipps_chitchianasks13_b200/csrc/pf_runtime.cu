@@ -182,7 +182,7 @@ pf::StepParams base_params(pf_handle* h, long long k, int mode) {
   p.counter = reinterpret_cast<unsigned int*>(h->scratch + kOffCounter);
   p.work = reinterpret_cast<unsigned int*>(h->scratch + kOffWork);
   p.record = record(h);
-  p.record_host = h->rec_host_dev;
+  p.record_host = std::getenv("PF_NO_MAPPED") ? nullptr : h->rec_host_dev;
   p.est_out = nullptr;
   p.dbg_src = nullptr;
   p.dbg_anc = nullptr;
