@@ -251,3 +251,31 @@ def test_full_size_sampled(P, orc, W, name, nj, m, N, t, topo, res):
     assert lw == wg.max() and idx == int(np.flatnonzero(wg == wg.max())[0])
     np.testing.assert_array_equal(x, sg[:, idx])
     g.close()
+
+
+def test_rmse_100_seeds_c1(P, orc, W):
+    # north_star: end-to-end tracking RMSE within 5 % of the oracle's over 100
+    # seeds (config C1: 2-link arm, 16 x 64, RWS, ring t = 1, 100 steps).
+    # With the fp32 contract the estimates are bit-identical, so the RMSEs agree exactly.
+    nj, T = 2, 100
+    rg, ro = [], []
+    for seed in range(100):
+        tr = W.make_trajectory(nj, T, seed)
+        g = P.ParticleFilter(tr["mu0"], tr["sigma0"], P.ArmModel(n_joints=nj), m=64, n_filters=16, t=1,
+                             topo="ring", resampler="rws", seed=seed)
+        o = orc.Filter(orc.Config(m=64, n_filters=16, t=1, topo="ring", resampler="rws", seed=seed),
+                       orc.Model(n_joints=nj), tr["mu0"], tr["sigma0"])
+        eg, eo = [], []
+        for k in range(1, T + 1):
+            g.step(tr["Z"][k], tr["U"][k - 1])
+            o.step(tr["Z"][k], tr["U"][k - 1])
+            truth = tr["X"][k][nj:nj + 2]
+            eg.append(np.hypot(*(g.estimate()[0][nj:nj + 2] - truth)))
+            eo.append(np.hypot(*(o.estimate()[0][nj:nj + 2] - truth)))
+        g.close()
+        rg.append(np.sqrt(np.mean(np.square(eg))))
+        ro.append(np.sqrt(np.mean(np.square(eo))))
+    mg, mo = float(np.mean(rg)), float(np.mean(ro))
+    assert abs(mg - mo) <= 0.05 * mo, (mg, mo)
+    np.testing.assert_array_equal(rg, ro)
+    assert mo < 0.25   # tracks the lemniscate (Fig.8)
