@@ -46,8 +46,11 @@ typedef enum {
   PF_EUNSUPPORTED = -6   /* (n_joints, m) combination not compiled           */
 } pf_status;
 
-/* Exchange scheme X (PAPER.md:18 Table I; :16 Fig.1; :20 §VI-E). */
-typedef enum { PF_TOPO_NONE = 0, PF_TOPO_RING = 1, PF_TOPO_TORUS2D = 2 } pf_topology;
+/* Exchange scheme X (PAPER.md:18 Table I; :16 Fig.1; :20 §VI-E): Ring and
+ * 2D Torus exchange t particles per neighbour pair; All-to-All — "each
+ * sub-filter supplies [t]. Then, all sub-filters read back the same t best
+ * particles from the supplied set" (§VI-E). */
+typedef enum { PF_TOPO_NONE = 0, PF_TOPO_RING = 1, PF_TOPO_TORUS2D = 2, PF_TOPO_ALL2ALL = 3 } pf_topology;
 /* Resampler (PAPER.md:18 §IV; :20–22 §VI-F). */
 typedef enum { PF_RESAMPLE_RWS = 0, PF_RESAMPLE_VOSE = 1 } pf_resampler;
 /* Model hooks (the paper separates "generic particle filtering from
@@ -109,7 +112,11 @@ typedef struct {
  * with neighbour ranks' entries before step k+1: ring — row n_local holds
  * global sub-filter (g0-1) mod N, row n_local+1 holds (g0+n_local) mod N;
  * torus — rows n_local + c hold grid row (r0-1) mod R, rows
- * n_local + C + c hold grid row (r1) mod R (c = column). */
+ * n_local + C + c hold grid row (r1) mod R (c = column).  All-to-All: the
+ * kernel writes this shard's best t of the pool into row n_local + rank
+ * (world > 1) or n_local (world == 1); with world > 1 the caller all-gathers
+ * rows [n_local, n_local + world) and calls pf_reduce_pool, which writes the
+ * global best t into row n_local + world — the row every sub-filter reads. */
 typedef struct {
   int64_t g0;            /* first global sub-filter of this shard                  */
   int64_t n_local;       /* local sub-filters                                      */
@@ -173,6 +180,12 @@ pf_status pf_record_ptr(pf_handle* h, float** record_dev, int32_t* record_floats
  * all-gather of every rank's record): picks the maximal key (exact,
  * order-free) and makes it this handle's estimate.  Asynchronous. */
 pf_status pf_reduce_records(pf_handle* h, const float* records_dev, int32_t count);
+
+/* All-to-All with world > 1: after the rows [n_local, n_local + world) of
+ * the last step's mailbox parity hold every rank's best t (all-gather),
+ * select the global best t (order key R6; exact) into row n_local + world.
+ * Asynchronous.  PF_ESTATE unless topo == PF_TOPO_ALL2ALL and world > 1. */
+pf_status pf_reduce_pool(pf_handle* h);
 
 /* Shard geometry and mailbox layout for halo exchange. */
 pf_status pf_get_shard(const pf_handle* h, pf_shard* out);

@@ -39,7 +39,7 @@
 extern "C" {
 #endif
 
-enum { ORC_TOPO_NONE = 0, ORC_TOPO_RING = 1, ORC_TOPO_TORUS2D = 2 };
+enum { ORC_TOPO_NONE = 0, ORC_TOPO_RING = 1, ORC_TOPO_TORUS2D = 2, ORC_TOPO_ALL2ALL = 3 };
 enum { ORC_RWS = 0, ORC_VOSE = 1 };
 
 /* Table I parameters: m, N, X, t; plus the RNG seed. */

@@ -18,7 +18,7 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(HERE, "liborc.so")
 SOURCES = [os.path.join(HERE, f) for f in ("orc.c", "orc_impl.inc", "orc.h")]
 
-TOPO = {"none": 0, "ring": 1, "torus": 2}
+TOPO = {"none": 0, "ring": 1, "torus": 2, "all2all": 3}
 RESAMPLER = {"rws": 0, "vose": 1}
 
 CFLAGS = ["-O2", "-std=c11", "-Wall", "-ffp-contract=off", "-fno-fast-math", "-fPIC", "-shared"]

@@ -14,14 +14,14 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(HERE, "libpf_b200.so")
 
 PF_OK, PF_EINVAL, PF_ENOMEM, PF_ECUDA, PF_ESTATE, PF_EUNSUPPORTED = 0, -1, -2, -3, -5, -6
-PF_TOPO_NONE, PF_TOPO_RING, PF_TOPO_TORUS2D = 0, 1, 2
+PF_TOPO_NONE, PF_TOPO_RING, PF_TOPO_TORUS2D, PF_TOPO_ALL2ALL = 0, 1, 2, 3
 PF_RESAMPLE_RWS, PF_RESAMPLE_VOSE = 0, 1
 PF_MODEL_ARM_PLANAR = 0
 PF_DEVICE_INPUTS = 1
 
 ENTRY_POINTS = [
     "pf_query_sizes", "pf_init", "pf_step", "pf_step_batch", "pf_estimate", "pf_record_ptr",
-    "pf_reduce_records", "pf_get_shard", "pf_get_particles", "pf_set_particles", "pf_debug_sample_weight",
+    "pf_reduce_records", "pf_reduce_pool", "pf_get_shard", "pf_get_particles", "pf_set_particles", "pf_debug_sample_weight",
     "pf_debug_resample", "pf_debug_exchange", "pf_set_trace", "pf_get_trace", "pf_destroy", "pf_strerror",
     "pf_last_error", "pf_supported", "pf_debug_math", "pf_debug_check_sqrt",
 ]
@@ -78,6 +78,7 @@ def lib() -> C.CDLL:
             "pf_estimate": [P, P, P, P],
             "pf_record_ptr": [P, P, P],
             "pf_reduce_records": [P, P, I32],
+            "pf_reduce_pool": [P],
             "pf_get_shard": [P, P],
             "pf_get_particles": [P, P, P, P],
             "pf_set_particles": [P, P, P, I64],
@@ -157,6 +158,10 @@ def pf_record_ptr(h) -> tuple[int, int]:
 
 def pf_reduce_records(h, records_dev, count: int) -> None:
     check(lib().pf_reduce_records(h, _ptr(records_dev), count), "pf_reduce_records")
+
+
+def pf_reduce_pool(h) -> None:
+    check(lib().pf_reduce_pool(h), "pf_reduce_pool")
 
 
 def pf_get_shard(h) -> pf_shard:

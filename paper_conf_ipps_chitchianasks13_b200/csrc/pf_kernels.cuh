@@ -39,7 +39,7 @@ namespace pf {
 typedef unsigned long long u64;
 
 enum : int { MODE_STEP = 0, MODE_PUBLISH = 1, MODE_EXCHANGE = 2, MODE_SAMPLE = 3 };
-enum : int { TOPO_NONE = 0, TOPO_RING = 1, TOPO_TORUS = 2 };
+enum : int { TOPO_NONE = 0, TOPO_RING = 1, TOPO_TORUS = 2, TOPO_A2A = 3 };
 enum : int { RES_RWS = 0, RES_VOSE = 1 };
 
 struct StepParams {
@@ -59,6 +59,8 @@ struct StepParams {
   long long* dbg_src;      // nullable [M_local] exchange sources (global index)
   int* dbg_anc;            // nullable [M_local] ancestors
   long long n_local, g0, n_global, R, C;
+  long long pool_row;      // All-to-All: the row every sub-filter reads (global best t)
+  long long pool_local_row;  // All-to-All: where the last CTA writes this shard's best t
   int t, tt, topo, deg;
   uint32_t k;
   int mode, first;
@@ -402,6 +404,7 @@ __device__ __forceinline__ void resample_group(const uint32_t (&q)[C::P], const 
 // are always local and up/down leave the shard only at its first/last row.
 __device__ __forceinline__ long long neighbor_row(const StepParams& P, long long g, int qi) {
   const long long N = P.n_global;
+  if (P.topo == TOPO_A2A) return P.pool_row;
   if (P.topo == TOPO_RING) {
     const long long q = qi == 0 ? (g == 0 ? N - 1 : g - 1) : (g == N - 1 ? 0 : g + 1);
     const long long loc = q - P.g0;
@@ -451,6 +454,45 @@ struct SamplePairs {
     if constexpr (QP + 1 < (D + 1) / 2) SamplePairs<NJ, QP + 1>::run(mc, hsu, x, gen, xo);
   }
 };
+
+// All-to-All pool (§VI-E): the best t of `count` mailbox entries
+// (entry e = row e / t, item e % t, E floats [logw, index bits, x]) by the
+// order key of R6, copied to out[0..t) in order.  Whole CTA; t rounds.
+template <int E>
+__device__ void pool_top_t(const StepParams& P, const float* mb, long long count, float* out) {
+  __shared__ u64 pool_red[33];
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5, nw = (blockDim.x + 31) >> 5;
+  u64 prev = ~0ull;
+  for (int jb = 0; jb < P.t; ++jb) {
+    u64 best = 0ull;
+    long long be = -1;
+    for (long long e = tid; e < count; e += blockDim.x) {
+      const long long row = e / P.t, jj = e - row * P.t;
+      const float* en = mb + (row * P.tt + jj) * E;
+      const u64 key = order_key(__ldcg(en), __float_as_uint(__ldcg(en + 1)));
+      if (key < prev && key > best) {
+        best = key;
+        be = e;
+      }
+    }
+    const u64 wbest = warp_max_u64(best);
+    if (lane == 0) pool_red[warp] = wbest;
+    __syncthreads();
+    if (warp == 0) {
+      const u64 v = warp_max_u64(lane < nw ? pool_red[lane] : 0ull);
+      if (lane == 0) pool_red[32] = v;
+    }
+    __syncthreads();
+    const u64 g = pool_red[32];
+    if (best == g && be >= 0) {   // unique owner (the index is part of the key)
+      const long long row = be / P.t, jj = be - row * P.t;
+      const float* en = mb + (row * P.tt + jj) * E;
+      for (int c = 0; c < E; ++c) out[jb * E + c] = __ldcg(en + c);
+    }
+    prev = g;
+    __syncthreads();
+  }
+}
 
 // ------------------------------------------------------------ the kernel
 template <class C>
@@ -840,6 +882,8 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
             for (int c = 0; c < 4; ++c) outs[o][c] = r[c];
       }
     }
+    if (P.topo == TOPO_A2A && P.t > 0 && mode != MODE_EXCHANGE)
+      pool_top_t<E>(P, P.mb_cur, P.n_local * P.t, P.mb_cur + P.pool_local_row * P.tt * E);
     if (tid == 0) {
       *P.key_next = 0ull;
       *P.counter = 0u;

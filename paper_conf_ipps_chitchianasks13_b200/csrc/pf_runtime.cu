@@ -90,13 +90,15 @@ pf_status validate(const pf_config* cfg, const pf_model_params* mp, Geometry* g)
   if (cfg->n_filters < 1 || cfg->t < 0 || cfg->world < 1 || cfg->rank < 0 || cfg->rank >= cfg->world)
     return PF_EINVAL;
   if (cfg->resampler != PF_RESAMPLE_RWS && cfg->resampler != PF_RESAMPLE_VOSE) return PF_EINVAL;
-  if (cfg->topo != PF_TOPO_NONE && cfg->topo != PF_TOPO_RING && cfg->topo != PF_TOPO_TORUS2D) return PF_EINVAL;
+  if (cfg->topo != PF_TOPO_NONE && cfg->topo != PF_TOPO_RING && cfg->topo != PF_TOPO_TORUS2D &&
+      cfg->topo != PF_TOPO_ALL2ALL)
+    return PF_EINVAL;
   if (!find_entry(mp->n_joints, m, cfg->resampler)) return PF_EUNSUPPORTED;
   g->nj = mp->n_joints;
   g->d = mp->n_joints + 4;
   g->m = m;
   g->N = cfg->n_filters;
-  g->deg = cfg->topo == PF_TOPO_RING ? 2 : cfg->topo == PF_TOPO_TORUS2D ? 4 : 0;
+  g->deg = cfg->topo == PF_TOPO_RING ? 2 : cfg->topo == PF_TOPO_TORUS2D ? 4 : cfg->topo == PF_TOPO_ALL2ALL ? 1 : 0;
   if (static_cast<long long>(g->deg) * cfg->t >= m && g->deg * cfg->t > 0) return PF_EINVAL;   // R19
   if (g->deg * cfg->t > 32) return PF_EINVAL;   // exchange list fits one warp (KMAX)
   g->tt = cfg->t > 0 ? cfg->t : 1;
@@ -122,7 +124,8 @@ pf_status validate(const pf_config* cfg, const pf_model_params* mp, Geometry* g)
     if (g->N % W != 0) return PF_EINVAL;
     g->n_local = g->N / W;
     g->g0 = cfg->rank * g->n_local;
-    g->n_ext = g->n_local + ((W > 1 && cfg->topo == PF_TOPO_RING) ? 2 : 0);
+    g->n_ext = g->n_local + ((W > 1 && cfg->topo == PF_TOPO_RING) ? 2 : 0) +
+               (cfg->topo == PF_TOPO_ALL2ALL ? (W > 1 ? W + 1 : 1) : 0);
   }
   g->M_local = g->n_local * m;
   g->ROW = static_cast<long long>(g->d + 1) * m;
@@ -191,6 +194,8 @@ pf::StepParams base_params(pf_handle* h, long long k, int mode) {
   p.n_global = h->g.N;
   p.R = h->g.R;
   p.C = h->g.C;
+  p.pool_row = h->g.n_local + (h->cfg.world > 1 ? h->cfg.world : 0);
+  p.pool_local_row = h->g.n_local + (h->cfg.world > 1 ? h->cfg.rank : 0);
   p.t = h->cfg.t;
   p.tt = h->g.tt;
   p.topo = h->cfg.topo;
@@ -241,6 +246,34 @@ __global__ void pf_init_kernel(float* parts, int m, long long M_local, uint32_t 
       if (c + 1 < d) blk[(c + 1) * m] = __fmaf_rn(s0[c + 1], z1, mu0[c + 1]);
     }
     blk[d * m] = 0.0f;
+  }
+}
+
+// All-to-All with world > 1: the global best t of the world gathered rows
+// [n_local, n_local + world) (t entries of E floats each) -> row out.
+__global__ void pf_reduce_pool_kernel(const float* rows, int world, int t, int tt, int E, float* out) {
+  const int lane = threadIdx.x;
+  pf::u64 prev = ~0ull;
+  for (int jb = 0; jb < t; ++jb) {
+    pf::u64 best = 0ull;
+    int be = -1;
+    for (int e = lane; e < world * t; e += 32) {
+      const int r = e / t, jj = e - r * t;
+      const float* en = rows + (static_cast<long long>(r) * tt + jj) * E;
+      const pf::u64 key = pf::order_key(en[0], __float_as_uint(en[1]));
+      if (key < prev && key > best) {
+        best = key;
+        be = e;
+      }
+    }
+    const pf::u64 g = pf::warp_max_u64(best);
+    if (best == g && be >= 0) {
+      const int r = be / t, jj = be - r * t;
+      const float* en = rows + (static_cast<long long>(r) * tt + jj) * E;
+      for (int c = 0; c < E; ++c) out[jb * E + c] = en[c];
+    }
+    prev = g;
+    __syncwarp();
   }
 }
 
@@ -453,6 +486,17 @@ pf_status pf_reduce_records(pf_handle* h, const float* records_dev, int32_t coun
   if (!h || !records_dev || count < 1) return PF_EINVAL;
   if (h->err != PF_OK) return h->err;
   pf_reduce_records_kernel<<<1, 32, 0, h->stream>>>(records_dev, count, 4 + h->g.d, record(h), h->rec_host_dev);
+  return sticky(h, cudaGetLastError());
+}
+
+pf_status pf_reduce_pool(pf_handle* h) {
+  if (!h) return PF_EINVAL;
+  if (h->err != PF_OK) return h->err;
+  if (h->cfg.topo != PF_TOPO_ALL2ALL || h->cfg.world < 2 || h->cfg.t < 1 || h->step < 1) return PF_ESTATE;
+  float* mb = mailbox_parity(h, h->step);
+  const long long rowf = static_cast<long long>(h->g.tt) * h->g.E;
+  pf_reduce_pool_kernel<<<1, 32, 0, h->stream>>>(mb + h->g.n_local * rowf, h->cfg.world, h->cfg.t, h->g.tt, h->g.E,
+                                                 mb + (h->g.n_local + h->cfg.world) * rowf);
   return sticky(h, cudaGetLastError());
 }
 

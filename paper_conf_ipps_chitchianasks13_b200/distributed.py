@@ -23,7 +23,7 @@ from dataclasses import dataclass
 import torch
 import torch.distributed as dist
 
-RING, TORUS = "ring", "torus"
+RING, TORUS, ALL2ALL = "ring", "torus", "all2all"
 
 
 @dataclass(frozen=True)
@@ -54,7 +54,8 @@ def shard_geometry(topo: str, n_filters: int, world: int, rank: int, R: int = 0,
         rows = R // world
         return rank * rows * C, rows * C, rows * C + (2 * C if world > 1 else 0)
     n_local = n_filters // world
-    return rank * n_local, n_local, n_local + (2 if (world > 1 and topo == RING) else 0)
+    extra = (2 if (world > 1 and topo == RING) else 0) + ((world + 1 if world > 1 else 1) if topo == ALL2ALL else 0)
+    return rank * n_local, n_local, n_local + extra
 
 
 def halo_plan(topo: str, n_filters: int, world: int, R: int = 0, C: int = 0) -> list[Transfer]:
@@ -107,6 +108,13 @@ def exchange_halos(mailbox_parity: torch.Tensor, plan: list[Transfer], rank: int
             w.wait()
 
 
+def gather_pool(mailbox_parity: torch.Tensor, n_local: int, rank: int, world: int, group=None) -> None:
+    """All-to-All: all-gather every rank's best-t row (row n_local + rank) into
+    rows [n_local, n_local + world) of one mailbox parity (in place)."""
+    rows = mailbox_parity[n_local:n_local + world]
+    dist.all_gather_into_tensor(rows.reshape(-1), rows[rank].reshape(-1).clone(), group=group)
+
+
 def loopback_exchange(mailboxes: list[torch.Tensor], plan: list[Transfer]) -> None:
     """The same plan between shards held by one process (e.g. on one GPU)."""
     for t in plan:
@@ -135,6 +143,10 @@ class DistributedFilter:
         self.pf.step(z, u)
         self.k += 1
         if self.world > 1:
+            if self.pf.topo == ALL2ALL and self.pf.t > 0:
+                gather_pool(self.pf.mailbox[self.k & 1], int(self.pf.shard.n_local), self.rank, self.world,
+                            self.group)
+                self.pf.reduce_pool()
             dist.all_gather_into_tensor(self._records, self.pf.record, group=self.group)
             self.pf.reduce_records(self._records)
 

@@ -13,7 +13,7 @@ import torch
 
 from . import binding as B
 
-TOPO = {"none": B.PF_TOPO_NONE, "ring": B.PF_TOPO_RING, "torus": B.PF_TOPO_TORUS2D}
+TOPO = {"none": B.PF_TOPO_NONE, "ring": B.PF_TOPO_RING, "torus": B.PF_TOPO_TORUS2D, "all2all": B.PF_TOPO_ALL2ALL}
 RESAMPLER = {"rws": B.PF_RESAMPLE_RWS, "vose": B.PF_RESAMPLE_VOSE}
 
 
@@ -117,6 +117,10 @@ class ParticleFilter:
 
     def reduce_records(self, records: torch.Tensor) -> None:
         B.pf_reduce_records(self.h, records.data_ptr(), records.shape[0])
+
+    def reduce_pool(self) -> None:
+        """All-to-All, world > 1: global best t from the gathered pool rows."""
+        B.pf_reduce_pool(self.h)
 
     def get_particles(self):
         s = np.zeros((self.d, self.M_local), np.float32)

@@ -50,6 +50,14 @@ def _worker(rank, world, port, cases, ret):
                 assert torch.all(mb[row] == float(gid)), (topo, N, rank, row, gid, mb[row].flatten()[:3])
             for row in range(n_local):
                 assert torch.all(mb[row] == float(g0 + row))
+        # All-to-All pool rows: every rank's best-t row gathered in place
+        g0, n_local, n_ext = Dd.shard_geometry("all2all", 4 * world, world, rank)
+        assert n_ext == n_local + world + 1
+        mb = torch.full((n_ext, 2, 5), -1.0)
+        mb[n_local + rank] = float(100 + rank)
+        Dd.gather_pool(mb, n_local, rank, world)
+        for r in range(world):
+            assert torch.all(mb[n_local + r] == float(100 + r))
         # estimate protocol: ordered key of every rank's best, all-gather, max
         rng = np.random.default_rng(7)
         w = np.round(rng.normal(-20, 5, 64 * world) * 2).astype(np.float32) / 2   # ties across ranks

@@ -82,7 +82,7 @@ def test_resample_bit_exact(P, orc, W, res, m, kind):
 
 @pytest.mark.parametrize("topo,N,m,t", [("ring", 16, 64, 1), ("ring", 8, 32, 3), ("torus", 16, 64, 2),
                                          ("torus", 8, 128, 1), ("ring", 2, 32, 1), ("torus", 4, 32, 1),
-                                         ("ring", 1, 32, 2)])
+                                         ("ring", 1, 32, 2), ("all2all", 8, 32, 3), ("all2all", 64, 64, 1)])
 def test_exchange_bit_exact(P, orc, W, topo, N, m, t):
     tr = W.make_trajectory(2, 4, 0)
     g = P.ParticleFilter(tr["mu0"], tr["sigma0"], P.ArmModel(n_joints=2), m=m, n_filters=N, t=t, topo=topo)
@@ -131,6 +131,8 @@ def test_full_filter_c1(P, orc, W):
     (5, 32, 32, 0, "none", "rws"),
     (28, 64, 8, 1, "ring", "vose"),
     (5, 1024, 4, 4, "torus", "rws"),
+    (5, 64, 16, 2, "all2all", "vose"),
+    (2, 256, 64, 1, "all2all", "rws"),
 ])
 def test_full_filter_variants(P, orc, W, nj, m, N, t, topo, res):
     _run_compare(P, orc, W, nj, m, N, 12, t=t, topo=topo, res=res, seed=nj * 1000 + m)
@@ -187,7 +189,8 @@ def test_step_batch_matches_streaming(P, W):
         assert est[k - 1, 2].item() == lw
 
 
-@pytest.mark.parametrize("topo,N,world", [("ring", 16, 2), ("torus", 16, 2), ("ring", 12, 4), ("torus", 64, 4)])
+@pytest.mark.parametrize("topo,N,world", [("ring", 16, 2), ("torus", 16, 2), ("ring", 12, 4), ("torus", 64, 4),
+                                          ("all2all", 16, 2), ("all2all", 24, 4)])
 def test_sharded_loopback_bit_identical(P, orc, W, topo, N, world):
     # world shards of one filter in one process on one GPU, halos exchanged
     # by the same plan the NCCL path uses: identical to the unsharded filter
@@ -196,18 +199,26 @@ def test_sharded_loopback_bit_identical(P, orc, W, topo, N, world):
     from paper_conf_ipps_chitchianasks13_b200 import distributed as Dd
     nj, m, T = 5, 64, 6
     tr = W.make_trajectory(nj, T, 4)
-    kw = dict(m=m, n_filters=N, t=1, topo=topo, resampler="vose", seed=99)
+    t = 2 if topo == "all2all" else 1
+    kw = dict(m=m, n_filters=N, t=t, topo=topo, resampler="vose", seed=99)
     shards = [P.ParticleFilter(tr["mu0"], tr["sigma0"], P.ArmModel(n_joints=nj), rank=r, world=world, **kw)
               for r in range(world)]
-    o = orc.Filter(orc.Config(m=m, n_filters=N, t=1, topo=topo, resampler="vose", seed=99),
+    o = orc.Filter(orc.Config(m=m, n_filters=N, t=t, topo=topo, resampler="vose", seed=99),
                    orc.Model(n_joints=nj), tr["mu0"], tr["sigma0"])
     plan = Dd.halo_plan(topo, N, world)
+    nl = int(shards[0].shard.n_local)
     recs = torch.zeros(world, 4 + nj + 4, device="cuda")
     for k in range(1, T + 1):
         if k > 1:
             Dd.loopback_exchange([s.mailbox[(k - 1) & 1] for s in shards], plan)
         for s in shards:
             s.step(tr["Z"][k], tr["U"][k - 1])
+        if topo == "all2all":   # the all-gather of every shard's best-t row, then the exact reduce
+            for r in range(world):
+                for s in shards:
+                    s.mailbox[k & 1][nl + r].copy_(shards[r].mailbox[k & 1][nl + r])
+            for s in shards:
+                s.reduce_pool()
         for r, s in enumerate(shards):
             recs[r] = s.record
         shards[0].reduce_records(recs)

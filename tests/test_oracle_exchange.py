@@ -73,3 +73,28 @@ def test_exchange_properties_brute_force(orc, W):
                 assert src[n][slot] == incoming[j]
             for slot in set(range(m)) - set(worst):
                 assert src[n][slot] == n * m + slot
+
+
+def test_exchange_golden_all2all(orc):
+    g = G["all2all"]
+    for t, key in [(1, "src_t1"), (2, "src_t2")]:
+        cfg = orc.Config(m=g["m"], n_filters=g["N"], t=t, topo="all2all")
+        np.testing.assert_array_equal(orc.exchange(cfg, g["logw"]), g[key])
+
+
+def test_all2all_brute_force(orc, W):
+    # every sub-filter's worst t slots receive the global best t of the pool
+    # of supplied particles (each sub-filter's best t), in order
+    for N, m, t in [(8, 16, 3), (5, 32, 1), (16, 8, 2)]:
+        cfg = orc.Config(m=m, n_filters=N, t=t, topo="all2all")
+        w = W.random_logw(N, m, N * m + t)
+        src = orc.exchange(cfg, w)
+        rank = lambda n: sorted(range(m), key=lambda i: (-w[n][i], i))
+        pool = [n * m + rank(n)[j] for n in range(N) for j in range(t)]
+        top = sorted(pool, key=lambda p: (-w.ravel()[p], p))[:t]
+        for n in range(N):
+            worst = rank(n)[::-1][:t]
+            for j, slot in enumerate(worst):
+                assert src[n][slot] == top[j]
+            for slot in set(range(m)) - set(worst):
+                assert src[n][slot] == n * m + slot

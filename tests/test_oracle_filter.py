@@ -118,7 +118,7 @@ def test_fp32_matches_fp64_accuracy(orc, W):
 def test_step_subset_equals_whole_filter(orc, W):
     # the one-sub-filter-at-a-time oracle used for full-size sampled checks
     # reproduces the whole-filter step exactly
-    for topo, res, t in [("ring", "rws", 1), ("torus", "vose", 2), ("none", "rws", 0)]:
+    for topo, res, t in [("ring", "rws", 1), ("torus", "vose", 2), ("none", "rws", 0), ("all2all", "rws", 2)]:
         cfg = orc.Config(m=32, n_filters=16, t=t, topo=topo, resampler=res, seed=5)
         md = orc.Model(n_joints=5)
         tr = W.make_trajectory(5, 10, 0)
