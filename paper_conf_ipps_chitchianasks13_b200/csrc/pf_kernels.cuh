@@ -882,8 +882,22 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
             for (int c = 0; c < 4; ++c) outs[o][c] = r[c];
       }
     }
-    if (P.topo == TOPO_A2A && P.t > 0 && mode != MODE_EXCHANGE)
-      pool_top_t<E>(P, P.mb_cur, P.n_local * P.t, P.mb_cur + P.pool_local_row * P.tt * E);
+    if (P.topo == TOPO_A2A && P.t > 0 && mode != MODE_EXCHANGE) {
+      float* pool = P.mb_cur + P.pool_local_row * P.tt * E;
+      if (P.t == 1) {   // the pool's best is the shard's best particle: the record just written
+        const u64 key = __ldcg(P.key_cur);
+        const uint32_t gidx = 0xFFFFFFFFu - static_cast<uint32_t>(key);
+        const long long col = static_cast<long long>(gidx) - P.g0 * M;
+        const float* blk = P.parts + (col / M) * C::ROW + (col % M);
+        if (tid < D) pool[2 + tid] = __ldcg(blk + tid * M);
+        if (tid == 0) {
+          pool[0] = unord_f32(static_cast<uint32_t>(key >> 32));
+          pool[1] = __uint_as_float(gidx);
+        }
+      } else {
+        pool_top_t<E>(P, P.mb_cur, P.n_local * P.t, pool);
+      }
+    }
     if (tid == 0) {
       *P.key_next = 0ull;
       *P.counter = 0u;

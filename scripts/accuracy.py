@@ -51,12 +51,12 @@ def main():
     seeds = list(range(a.seeds))
     grid = []
     # Fig.6: exchange scheme x number of sub-filters x sub-filter size (t = 1)
-    for topo in ["ring", "torus"]:
+    for topo in ["ring", "torus", "all2all"]:
         for N in ([16, 256] if a.quick else [16, 64, 256, 1024]):
             for m in ([64] if a.quick else [32, 64, 128, 256]):
                 grid.append(("fig6", 5, m, N, topo, 1, "rws"))
     # Fig.7: particles per exchange (t = 0, 1, 2, 4; 64 x 64 ring and torus)
-    for topo in ["ring", "torus"]:
+    for topo in ["ring", "torus", "all2all"]:
         for t in [0, 1, 2, 4]:
             grid.append(("fig7", 5, 64, 64, topo, t, "rws"))
     # Fig.9: distributed vs centralized with equal particle count (a single

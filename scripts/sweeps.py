@@ -45,7 +45,7 @@ if __name__ == "__main__":
         for m in [32, 64, 128, 256, 512, 1024]:
             run("m", 5, m, (1 << 22) // m)
     if "t" in which:       # Fig.7 / C3: exchange count at 4M (ring and torus)
-        for topo in ["ring", "torus"]:
+        for topo in ["ring", "torus", "all2all"]:
             for t in [0, 1, 2, 4]:
                 run("t", 5, 256, 16384, topo=topo, t=t)
     if "dim" in which:     # Fig.4c / C4: state dimension
