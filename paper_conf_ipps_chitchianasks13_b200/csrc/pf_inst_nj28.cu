@@ -13,7 +13,6 @@ const KernelEntry kEntriesNJ28[] = {
     PF_LARGE_D_ENTRIES(28, 0), PF_LARGE_D_ENTRIES(28, 1),
     PF_ENTRY(28, 256, 0, 8, 1, 1, 1, 3), PF_ENTRY(28, 256, 0, 4, 1, 1, 1, 4), PF_ENTRY(28, 256, 0, 8, 1, 2, 1, 3),
     PF_ENTRY(28, 256, 1, 8, 1, 1, 1, 3), PF_ENTRY(28, 256, 1, 4, 1, 1, 1, 4),
-    PF_ENTRY_E(28, 256, 0, 8, 1, 1, 1, 4, 1), PF_ENTRY_E(28, 256, 1, 8, 1, 1, 1, 4, 1),
 };
 const int kNumEntriesNJ28 = sizeof(kEntriesNJ28) / sizeof(kEntriesNJ28[0]);
 }  // namespace pf

@@ -62,6 +62,7 @@ struct StepParams {
   long long pool_row;      // All-to-All: the row every sub-filter reads (global best t)
   long long pool_local_row;  // All-to-All: where the last CTA writes this shard's best t
   int t, tt, topo, deg;
+  uint32_t t_inv;          // ceil(2^16 / t): lane / t = (lane * t_inv) >> 16 for lane < 2^16 / t
   uint32_t k;
   int mode, first;
   uint32_t rk[20];         // Philox round keys (key0 + r W0, key1 + r W1), r = 0..9
@@ -617,9 +618,18 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
       }
       wmax = __reduce_max_sync(0xFFFFFFFFu, wmax);
       // incoming item j = (neighbour j / t, its j % t-th best): mailbox offset
-      if (G.lane < K) {
-        const int qi = G.lane / P.t;
-        woff[G.lane] = static_cast<int>((neighbor_row(P, gsf, qi) * P.tt + (G.lane - qi * P.t)) * E);
+      // (its log-weight, loaded now, gives the incoming maximum without a
+      // dependent shared-memory read after the copy)
+      uint32_t in_max = 0;
+      {
+        uint32_t in_o = 0;
+        if (G.lane < K) {
+          const int qi = static_cast<int>((static_cast<uint32_t>(G.lane) * P.t_inv) >> 16);   // lane / t
+          const int off = static_cast<int>((neighbor_row(P, gsf, qi) * P.tt + (G.lane - qi * P.t)) * E);
+          woff[G.lane] = off;
+          in_o = ord_f32(P.mb_prev[off]);
+        }
+        in_max = __reduce_max_sync(0xFFFFFFFFu, in_o);
       }
       u64 my_cand = ~0ull;
 #pragma unroll 1
@@ -697,8 +707,7 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
       gsync<GW>(g);
       // post-exchange max = max(pre-exchange max, incoming): the pre-exchange
       // maximum value survives because deg*t < m (R19)
-#pragma unroll 1
-      for (int j = 0; j < K; ++j) lmax_o = max(lmax_o, ord_f32(ws[wlist[j]]));
+      lmax_o = max(lmax_o, in_max);
 #pragma unroll
       for (int j = 0; j < PP; ++j)
         if ((excl >> j) & 1u) lw[j] = ws[C::slot(G.t, j)];

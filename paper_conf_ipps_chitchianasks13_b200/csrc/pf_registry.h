@@ -17,6 +17,7 @@ struct StepParams;
 struct KernelEntry {
   int nj, m, res;
   int gw, s, nstage, unr, minb;   // warps per group, groups per CTA, TMA stages, sample unroll, min CTAs/SM
+  int large;                      // preferred when the shard has >= kLargeNLocal sub-filters
   cudaError_t (*prepare)(int* blocks_per_sm);
   cudaError_t (*launch)(const StepParams& p, int grid, cudaStream_t s);
   cudaError_t (*resample_debug)(const uint32_t* q, const uint32_t* ua, const uint32_t* ub, int* anc,
@@ -41,6 +42,7 @@ extern const int kNumEntriesNJ28;
    NST,                                                                                                   \
    UNR,                                                                                                   \
    MINB,                                                                                                  \
+   0,                                                                                                     \
    &StepKernel<KCfg<NJ, M, RES, GW, S, NST, UNR, MINB>>::prepare,                                               \
    &StepKernel<KCfg<NJ, M, RES, GW, S, NST, UNR, MINB>>::launch,                                                \
    &StepKernel<KCfg<NJ, M, RES, GW, S, NST, UNR, MINB>>::resample_debug,                                        \
@@ -57,9 +59,9 @@ extern const int kNumEntriesNJ28;
 #define PF_LATENCY_ENTRIES(NJ, RES)                                                                  \
   PF_ENTRY(NJ, 64, RES, 2, 4, 1, 1, 3), PF_ENTRY(NJ, 128, RES, 4, 2, 1, 1, 3),                      \
       PF_ENTRY(NJ, 256, RES, 8, 1, 1, 1, 3)
-#define PF_ENTRY_E(NJ, M, RES, GW, S, NST, UNR, MINB, EARLY)                                      \
-  {NJ, M, RES, GW, S, NST, UNR, MINB,                                                                \
-   &StepKernel<KCfg<NJ, M, RES, GW, S, NST, UNR, MINB, EARLY>>::prepare,                             \
-   &StepKernel<KCfg<NJ, M, RES, GW, S, NST, UNR, MINB, EARLY>>::launch,                              \
-   &StepKernel<KCfg<NJ, M, RES, GW, S, NST, UNR, MINB, EARLY>>::resample_debug,                      \
-   StepKernel<KCfg<NJ, M, RES, GW, S, NST, UNR, MINB, EARLY>>::smem()}
+#define PF_ENTRY_LARGE(NJ, M, RES, GW, S, NST, UNR, MINB)                                           \
+  {NJ, M, RES, GW, S, NST, UNR, MINB, 1,                                                             \
+   &StepKernel<KCfg<NJ, M, RES, GW, S, NST, UNR, MINB>>::prepare,                                    \
+   &StepKernel<KCfg<NJ, M, RES, GW, S, NST, UNR, MINB>>::launch,                                     \
+   &StepKernel<KCfg<NJ, M, RES, GW, S, NST, UNR, MINB>>::resample_debug,                             \
+   StepKernel<KCfg<NJ, M, RES, GW, S, NST, UNR, MINB>>::smem()}

@@ -59,6 +59,17 @@ const pf::KernelEntry* find_entry(int nj, int m, int res) {
   return first;
 }
 
+// Large shards take the entry flagged `large` when one is compiled.
+constexpr long long kLargeNLocal = 8192;
+const pf::KernelEntry* large_entry(int nj, int m, int res) {
+  for (int ti = 0; ti < 3; ++ti) {
+    const Table t = tables(ti);
+    for (int i = 0; i < t.n; ++i)
+      if (t.e[i].nj == nj && t.e[i].m == m && t.e[i].res == res && t.e[i].large) return &t.e[i];
+  }
+  return nullptr;
+}
+
 // Small problems (too few sub-filters to keep the default mapping's groups
 // busy) are latency-bound: take the matching entry with the fewest particles
 // per thread.  PF_VARIANT, when set, wins.
@@ -197,6 +208,7 @@ pf::StepParams base_params(pf_handle* h, long long k, int mode) {
   p.pool_row = h->g.n_local + (h->cfg.world > 1 ? h->cfg.world : 0);
   p.pool_local_row = h->g.n_local + (h->cfg.world > 1 ? h->cfg.rank : 0);
   p.t = h->cfg.t;
+  p.t_inv = h->cfg.t > 0 ? (65536u + static_cast<uint32_t>(h->cfg.t) - 1u) / static_cast<uint32_t>(h->cfg.t) : 0u;
   p.tt = h->g.tt;
   p.topo = h->cfg.topo;
   p.deg = h->g.deg;
@@ -372,6 +384,16 @@ pf_status pf_init(const pf_config* cfg, const pf_model_params* model, const pf_b
   if (e != cudaSuccess) {
     pf_destroy(h);
     return PF_ECUDA;
+  }
+  if (!std::getenv("PF_VARIANT") && g.n_local >= kLargeNLocal) {
+    const pf::KernelEntry* le = large_entry(g.nj, g.m, cfg->resampler);
+    if (le && le != h->ke) {
+      int b2 = 0;
+      if (le->prepare(&b2) == cudaSuccess && b2 >= 1) {
+        h->ke = le;
+        bps = b2;
+      }
+    }
   }
   // fewer sub-filters than a quarter of the default mapping's groups: switch
   // to the lowest-latency mapping (more threads per sub-filter)
