@@ -290,3 +290,41 @@ def test_rmse_100_seeds_c1(P, orc, W):
     assert abs(mg - mo) <= 0.05 * mo, (mg, mo)
     np.testing.assert_array_equal(rg, ro)
     assert mo < 0.25   # tracks the lemniscate (Fig.8)
+
+
+@pytest.mark.parametrize("nj,m,N,t,topo,res,rows,cols", [
+    (5, 64, 16, 1, "torus", "rws", 2, 8),      # non-square torus
+    (5, 64, 16, 2, "torus", "vose", 8, 2),
+    (2, 32, 1, 1, "ring", "rws", 0, 0),       # one sub-filter: both ring neighbours are itself
+    (2, 32, 1, 3, "all2all", "vose", 0, 0),   # one sub-filter receiving its own best back
+    (5, 32, 4, 7, "torus", "rws", 0, 0),      # deg*t = 28 = m - 4 (R19 bound)
+    (5, 1024, 4, 8, "torus", "vose", 0, 0),   # deg*t = 32 = KMAX
+    (28, 32, 8, 0, "none", "rws", 0, 0),      # independent sub-filters
+])
+def test_edge_configs(P, orc, W, nj, m, N, t, topo, res, rows, cols):
+    tr = W.make_trajectory(nj, 8, 6)
+    kw = dict(m=m, n_filters=N, t=t, topo=topo, resampler=res, seed=(1 << 40) + 17, torus_rows=rows,
+              torus_cols=cols)
+    g = P.ParticleFilter(tr["mu0"], tr["sigma0"], P.ArmModel(n_joints=nj), **kw)
+    o = orc.Filter(orc.Config(**kw), orc.Model(n_joints=nj), tr["mu0"], tr["sigma0"])
+    for k in range(1, 7):
+        g.step(tr["Z"][k], tr["U"][k - 1])
+        o.step(tr["Z"][k], tr["U"][k - 1])
+        assert g.estimate()[2] == o.estimate()[2]
+    np.testing.assert_array_equal(g.get_particles()[0], o.get()[0])
+
+
+def test_error_behaviour(P, W):
+    from paper_conf_ipps_chitchianasks13_b200 import binding as B
+    tr = W.make_trajectory(2, 4, 0)
+    g = P.ParticleFilter(tr["mu0"], tr["sigma0"], P.ArmModel(n_joints=2), m=64, n_filters=4)
+    x = np.zeros(6, np.float32)
+    assert B.lib().pf_estimate(g.h, x.ctypes.data, None, None) == B.PF_ESTATE    # before the first step
+    assert B.lib().pf_reduce_pool(g.h) == B.PF_ESTATE                          # not All-to-All
+    assert B.lib().pf_step(g.h, None, None) == B.PF_EINVAL
+    assert B.lib().pf_destroy(None) == B.PF_OK
+    g.step(tr["Z"][1], tr["U"][0])
+    assert B.lib().pf_estimate(g.h, x.ctypes.data, None, None) == B.PF_OK
+    assert B.pf_last_error(g.h) == B.PF_OK
+    with pytest.raises(B.PFError):
+        P.ParticleFilter(tr["mu0"], tr["sigma0"], P.ArmModel(n_joints=3), m=64, n_filters=4)   # not compiled
