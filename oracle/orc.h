@@ -135,6 +135,12 @@ int orc_s_set(orc_s_filter* f, const float* state, const float* logw, int64_t st
 int orc_s_trace(const orc_s_filter* f, int64_t* src, int32_t* ancestors);
 void orc_s_destroy(orc_s_filter* f);
 
+/* Centralized filter (n_filters == 1): step k >= 2 for the listed slots only
+ * (normalise over all M, resample, sample, weight).  out_state [d][n]. */
+int orc_s_central_slots(const orc_config* cfg, const orc_model* md, const float* state, const float* logw,
+                        int64_t k, const float* z, const float* u, const int64_t* slots, int64_t n,
+                        float* out_state, float* out_logw);
+
 /* One step k >= 2 for the listed sub-filters only, from the full weighted
  * set of step k-1 (state [d][M], logw [M]) — exchange, normalise, resample,
  * sample, weight, one sub-filter at a time.  out_state [d][n_sub*m],

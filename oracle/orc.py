@@ -88,6 +88,7 @@ def lib():
             "orc_s_trace": (C.c_int, [P, P, P]),
             "orc_s_destroy": (None, [P]),
             "orc_s_step_subset": (C.c_int, [P, P, P, P, C.c_int64, P, P, P, C.c_int64, P, P]),
+            "orc_s_central_slots": (C.c_int, [P, P, P, P, C.c_int64, P, P, P, C.c_int64, P, P]),
             "orc_d_create": (P, [P, P, P, P]),
             "orc_d_step": (C.c_int, [P, P, P]),
             "orc_d_estimate": (C.c_int, [P, P, P, P]),
@@ -316,6 +317,21 @@ def step_subset(cfg: Config, model: Model, state, logw, k: int, z, u, subs):
                                  len(sb), _p(out_s), _p(out_w))
     if rc:
         raise ValueError(f"orc_s_step_subset failed: {rc}")
+    return out_s, out_w
+
+
+def central_slots(cfg: Config, model: Model, state, logw, k: int, z, u, slots):
+    """Centralized filter: step k of the listed slots from the weighted set of
+    step k-1: returns (state [d][len(slots)], logw [len(slots)])."""
+    st, lw = _f32(state), _f32(logw)
+    sl = np.ascontiguousarray(slots, np.int64)
+    out_s = np.zeros((model.d, len(sl)), np.float32)
+    out_w = np.zeros(len(sl), np.float32)
+    cc, mc = cfg.c(), model.c()
+    rc = lib().orc_s_central_slots(C.byref(cc), C.byref(mc), _p(st), _p(lw), k, _p(_f32(z)), _p(_f32(u)), _p(sl),
+                                   len(sl), _p(out_s), _p(out_w))
+    if rc:
+        raise ValueError(f"orc_s_central_slots failed: {rc}")
     return out_s, out_w
 
 

@@ -1,0 +1,41 @@
+// pf_central.h — launch interface of the centralized filter (pf_central.cu).
+#pragma once
+#include <cuda_runtime.h>
+
+#include <cstdint>
+
+#include "pf_device.cuh"
+
+namespace pf {
+
+constexpr int kCentralTile = 4096;   // particles per scan tile (M must be a multiple)
+
+struct CentralParams {
+  ArmConsts mc;
+  const float* in;          // [D+1][M] weighted set of step k-1 (buffer (k-1)&1)
+  float* out;               // [D+1][M] step k (buffer k&1)
+  long long M;
+  unsigned long long* cl;   // [M] per-tile inclusive sums of q
+  unsigned long long* tile_sum;    // [M / tile]
+  unsigned long long* tile_incl;   // [M / tile] inclusive prefix of the tile sums
+  const float* z;           // device or nullptr (zin)
+  const float* u;
+  float zin[32];
+  float uin[32];
+  unsigned long long* key_cur;
+  unsigned long long* key_next;
+  unsigned int* counter;
+  const float* record_prev;   // estimate record of step k-1 (its key gives l_max)
+  float* record;
+  float* est_out;
+  float* record_host;
+  uint32_t rk[20];
+  uint32_t k;
+  int first;     // k == 1 (or the sample-only test hook): no resampling
+  int publish;   // only the argmax / record of the set in `in` (checkpoint restore)
+};
+
+cudaError_t central_step(int nj, const CentralParams& c, int grid, cudaStream_t s);
+int central_grid(int nj, int sms);
+
+}  // namespace pf

@@ -12,6 +12,7 @@
 #include <new>
 
 #include "../../include/pf.h"
+#include "pf_central.h"
 #include "pf_kernels.cuh"
 #include "pf_registry.h"
 
@@ -88,6 +89,8 @@ const pf::KernelEntry* latency_entry(int nj, int m, int res) {
 struct Geometry {
   int nj, d, m, deg, tt, E;
   long long N, R, C, n_local, g0, n_ext, M_local, ROW;
+  bool central;   // one filter of m > 1024 particles, resampled globally (pf_central.cu)
+  long long tiles;
 };
 
 pf_status validate(const pf_config* cfg, const pf_model_params* mp, Geometry* g) {
@@ -97,9 +100,32 @@ pf_status validate(const pf_config* cfg, const pf_model_params* mp, Geometry* g)
       !(mp->sigma_pos >= 0.0f) || !(mp->sigma_vel >= 0.0f))
     return PF_EINVAL;
   const int m = cfg->m;
-  if (m < 32 || m > 1024 || (m & (m - 1)) != 0) return PF_EINVAL;
   if (cfg->n_filters < 1 || cfg->t < 0 || cfg->world < 1 || cfg->rank < 0 || cfg->rank >= cfg->world)
     return PF_EINVAL;
+  // Centralized filter (NEXT-2): a single filter of M > 1024 particles.
+  g->central = cfg->n_filters == 1 && m > 1024;
+  if (g->central) {
+    if (m % pf::kCentralTile != 0 || m > (1 << 26) || cfg->world != 1) return PF_EINVAL;
+    if (cfg->topo != PF_TOPO_NONE && cfg->t != 0) return PF_EINVAL;
+    if (cfg->resampler != PF_RESAMPLE_RWS) return PF_EUNSUPPORTED;
+    if (mp->n_joints != 2 && mp->n_joints != 5 && mp->n_joints != 28) return PF_EUNSUPPORTED;
+    g->nj = mp->n_joints;
+    g->d = mp->n_joints + 4;
+    g->m = m;
+    g->N = 1;
+    g->deg = 0;
+    g->tt = 1;
+    g->E = g->d + 2;
+    g->R = g->C = 0;
+    g->n_local = 1;
+    g->g0 = 0;
+    g->n_ext = 1;
+    g->M_local = m;
+    g->ROW = static_cast<long long>(g->d + 1) * m;
+    g->tiles = m / pf::kCentralTile;
+    return PF_OK;
+  }
+  if (m < 32 || m > 1024 || (m & (m - 1)) != 0) return PF_EINVAL;
   if (cfg->resampler != PF_RESAMPLE_RWS && cfg->resampler != PF_RESAMPLE_VOSE) return PF_EINVAL;
   if (cfg->topo != PF_TOPO_NONE && cfg->topo != PF_TOPO_RING && cfg->topo != PF_TOPO_TORUS2D &&
       cfg->topo != PF_TOPO_ALL2ALL)
@@ -233,8 +259,52 @@ void host_inputs(pf_handle* h, pf::StepParams& p, const float* z, const float* u
   std::memcpy(p.uin, u, sizeof(float) * h->g.nj);
 }
 
+// Centralized filter: particle buffers ping-pong ([2][D+1][M]), then the
+// per-particle tile sums (u64 [M]) and two u64 arrays of tile totals.
+size_t central_bytes(const Geometry& g) {
+  return sizeof(float) * 2 * g.ROW + sizeof(u64) * (g.M_local + 2 * g.tiles);
+}
+// weighted set of step k lives in particle buffer (central: k & 1; else the only one)
+float* set_of_step(pf_handle* h, long long k) { return h->parts + (h->g.central ? (k & 1) * h->g.ROW : 0); }
+
+pf::CentralParams central_params(pf_handle* h, long long k) {
+  pf::CentralParams c;
+  std::memset(&c, 0, sizeof(c));
+  c.mc = h->mc;
+  c.in = set_of_step(h, k - 1);
+  c.out = set_of_step(h, k);
+  c.M = h->g.M_local;
+  u64* aux = reinterpret_cast<u64*>(h->parts + 2 * h->g.ROW);
+  c.cl = aux;
+  c.tile_sum = aux + h->g.M_local;
+  c.tile_incl = aux + h->g.M_local + h->g.tiles;
+  c.key_cur = keys(h) + (k & 1);
+  c.key_next = keys(h) + ((k + 1) & 1);
+  c.counter = reinterpret_cast<unsigned int*>(h->scratch + kOffCounter);
+  c.record_prev = record(h);
+  c.record = record(h);
+  c.record_host = std::getenv("PF_NO_MAPPED") ? nullptr : h->rec_host_dev;
+  const uint32_t key0 = static_cast<uint32_t>(h->cfg.seed), key1 = static_cast<uint32_t>(h->cfg.seed >> 32);
+  for (int r = 0; r < 10; ++r) {
+    c.rk[2 * r] = key0 + static_cast<uint32_t>(r) * 0x9E3779B9u;
+    c.rk[2 * r + 1] = key1 + static_cast<uint32_t>(r) * 0xBB67AE85u;
+  }
+  c.k = static_cast<uint32_t>(k);
+  c.first = k == 1 ? 1 : 0;
+  return c;
+}
+
 pf_status launch(pf_handle* h, const pf::StepParams& p) {
   return sticky(h, h->ke->launch(p, h->grid, h->stream));
+}
+pf_status launch_central(pf_handle* h, const pf::CentralParams& c) {
+  return sticky(h, pf::central_step(h->g.nj, c, h->grid, h->stream));
+}
+void host_inputs(pf_handle* h, pf::CentralParams& c, const float* z, const float* u) {
+  c.z = nullptr;
+  c.u = nullptr;
+  std::memcpy(c.zin, z, sizeof(float) * (h->g.nj + 2));
+  std::memcpy(c.uin, u, sizeof(float) * h->g.nj);
 }
 
 __global__ void pf_init_kernel(float* parts, int m, long long M_local, uint32_t p0, int d, const float* mu0,
@@ -318,8 +388,8 @@ __global__ void pf_reduce_records_kernel(const float* recs, int count, int rec_f
 
 // host [d][M_local] rows <-> device blocked [n_local][d+1][m]: row c of the
 // host array maps to row c of every block (cudaMemcpy2D, pitch = block size).
-cudaError_t rows_to_device(pf_handle* h, const float* host, int row0, int nrows);
-cudaError_t rows_to_host(pf_handle* h, float* host, int row0, int nrows);
+cudaError_t rows_to_device(pf_handle* h, float* base, const float* host, int row0, int nrows);
+cudaError_t rows_to_host(pf_handle* h, const float* base, float* host, int row0, int nrows);
 
 template <typename T>
 struct DevBuf {
@@ -339,7 +409,7 @@ pf_status pf_query_sizes(const pf_config* cfg, const pf_model_params* model, pf_
   Geometry g;
   const pf_status s = validate(cfg, model, &g);
   if (s != PF_OK || !out) return s != PF_OK ? s : PF_EINVAL;
-  out->state = sizeof(float) * g.ROW * g.n_local;
+  out->state = g.central ? central_bytes(g) : sizeof(float) * g.ROW * g.n_local;
   out->mailbox = sizeof(float) * 2 * g.n_ext * g.tt * g.E;
   out->scratch = kScratchBytes;
   return PF_OK;
@@ -371,12 +441,18 @@ pf_status pf_init(const pf_config* cfg, const pf_model_params* model, const pf_b
   h->scratch = static_cast<unsigned char*>(buffers->scratch);
   h->stream = static_cast<cudaStream_t>(cuda_stream);
   h->step = 0;
-  h->ke = find_entry(g.nj, g.m, cfg->resampler);
+  h->ke = g.central ? nullptr : find_entry(g.nj, g.m, cfg->resampler);
   h->err = PF_OK;
   int dev = 0, sms = 0, bps = 0;
   cudaError_t e = cudaGetDevice(&dev);
   if (e == cudaSuccess) e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-  if (e == cudaSuccess) e = h->ke->prepare(&bps);
+  if (e == cudaSuccess && g.central) {
+    bps = 1;
+    h->grid = pf::central_grid(g.nj, sms);
+    if (h->grid < 1) e = cudaErrorInvalidConfiguration;
+  } else if (e == cudaSuccess) {
+    e = h->ke->prepare(&bps);
+  }
   if (e == cudaSuccess && bps < 1) e = cudaErrorInvalidConfiguration;
   if (e == cudaSuccess)
     e = cudaHostAlloc(reinterpret_cast<void**>(&h->rec_host), sizeof(float) * 64, cudaHostAllocMapped);
@@ -385,7 +461,7 @@ pf_status pf_init(const pf_config* cfg, const pf_model_params* model, const pf_b
     pf_destroy(h);
     return PF_ECUDA;
   }
-  if (!std::getenv("PF_VARIANT") && g.n_local >= kLargeNLocal) {
+  if (!g.central && !std::getenv("PF_VARIANT") && g.n_local >= kLargeNLocal) {
     const pf::KernelEntry* le = large_entry(g.nj, g.m, cfg->resampler);
     if (le && le != h->ke) {
       int b2 = 0;
@@ -397,7 +473,7 @@ pf_status pf_init(const pf_config* cfg, const pf_model_params* model, const pf_b
   }
   // fewer sub-filters than a quarter of the default mapping's groups: switch
   // to the lowest-latency mapping (more threads per sub-filter)
-  if (!std::getenv("PF_VARIANT") && g.n_local * 4 <= static_cast<long long>(bps) * sms * h->ke->s) {
+  if (!g.central && !std::getenv("PF_VARIANT") && g.n_local * 4 <= static_cast<long long>(bps) * sms * h->ke->s) {
     const pf::KernelEntry* le = latency_entry(g.nj, g.m, cfg->resampler);
     if (le && le != h->ke) {
       int b2 = 0;
@@ -407,9 +483,11 @@ pf_status pf_init(const pf_config* cfg, const pf_model_params* model, const pf_b
       }
     }
   }
-  const long long ctas_needed = (g.n_local + h->ke->s - 1) / h->ke->s;
-  const long long grid = static_cast<long long>(bps) * sms;
-  h->grid = static_cast<int>(grid < ctas_needed ? grid : ctas_needed);
+  if (!g.central) {
+    const long long ctas_needed = (g.n_local + h->ke->s - 1) / h->ke->s;
+    const long long grid = static_cast<long long>(bps) * sms;
+    h->grid = static_cast<int>(grid < ctas_needed ? grid : ctas_needed);
+  }
   // scratch: zero keys / counter; prior parameters
   float prior[128];
   std::memset(prior, 0, sizeof(prior));
@@ -441,6 +519,18 @@ pf_status pf_step(pf_handle* h, const float* z_k, const float* u_km1) {
   if (!h || !z_k || !u_km1) return PF_EINVAL;
   if (h->err != PF_OK) return h->err;
   const long long k = h->step + 1;
+  if (h->g.central) {
+    pf::CentralParams c = central_params(h, k);
+    if (h->cfg.flags & PF_DEVICE_INPUTS) {
+      c.z = z_k;
+      c.u = u_km1;
+    } else {
+      host_inputs(h, c, z_k, u_km1);
+    }
+    const pf_status s = launch_central(h, c);
+    if (s == PF_OK) h->step = k;
+    return s;
+  }
   pf::StepParams p = base_params(h, k, pf::MODE_STEP);
   if (h->cfg.flags & PF_DEVICE_INPUTS) {
     p.z = z_k;
@@ -464,6 +554,16 @@ pf_status pf_step_batch(pf_handle* h, int32_t T, const float* zs, const float* u
   const int nj = h->g.nj;
   for (int32_t s = 0; s < T; ++s) {
     const long long k = h->step + 1;
+    if (h->g.central) {
+      pf::CentralParams c = central_params(h, k);
+      c.z = zs + static_cast<long long>(s) * (nj + 2);
+      c.u = us + static_cast<long long>(s) * nj;
+      c.est_out = est ? est + static_cast<long long>(s) * (4 + h->g.d) : nullptr;
+      const pf_status st = launch_central(h, c);
+      if (st != PF_OK) return st;
+      h->step = k;
+      continue;
+    }
     pf::StepParams p = base_params(h, k, pf::MODE_STEP);
     p.z = zs + static_cast<long long>(s) * (nj + 2);
     p.u = us + static_cast<long long>(s) * nj;
@@ -541,8 +641,8 @@ pf_status pf_get_particles(pf_handle* h, float* state_host, float* logw_host, in
   if (h->err != PF_OK) return h->err;
   cudaError_t e = cudaStreamSynchronize(h->stream);
   if (e == cudaSuccess)
-    e = rows_to_host(h, state_host, 0, h->g.d);
-  if (e == cudaSuccess && logw_host) e = rows_to_host(h, logw_host, h->g.d, 1);
+    e = rows_to_host(h, set_of_step(h, h->step), state_host, 0, h->g.d);
+  if (e == cudaSuccess && logw_host) e = rows_to_host(h, set_of_step(h, h->step), logw_host, h->g.d, 1);
   if (step) *step = h->step;
   return sticky(h, e);
 }
@@ -550,6 +650,12 @@ pf_status pf_get_particles(pf_handle* h, float* state_host, float* logw_host, in
 static pf_status publish(pf_handle* h, long long step) {
   cudaError_t e = cudaMemsetAsync(keys(h), 0, 2 * sizeof(u64), h->stream);
   if (e != cudaSuccess) return sticky(h, e);
+  if (h->g.central) {
+    pf::CentralParams c = central_params(h, step);
+    c.in = set_of_step(h, step);
+    c.publish = 1;
+    return launch_central(h, c);
+  }
   pf::StepParams p = base_params(h, step, pf::MODE_PUBLISH);
   return launch(h, p);
 }
@@ -559,8 +665,8 @@ pf_status pf_set_particles(pf_handle* h, const float* state_host, const float* l
   if (h->err != PF_OK) return h->err;
   cudaError_t e = cudaStreamSynchronize(h->stream);
   if (e == cudaSuccess)
-    e = rows_to_device(h, state_host, 0, h->g.d);
-  if (e == cudaSuccess) e = rows_to_device(h, logw_host, h->g.d, 1);
+    e = rows_to_device(h, set_of_step(h, step), state_host, 0, h->g.d);
+  if (e == cudaSuccess) e = rows_to_device(h, set_of_step(h, step), logw_host, h->g.d, 1);
   if (e != cudaSuccess) return sticky(h, e);
   pf_status s = publish(h, step);
   if (s != PF_OK) return s;
@@ -575,18 +681,26 @@ pf_status pf_debug_sample_weight(pf_handle* h, const float* state_in, const floa
   if (h->cfg.world != 1) return PF_ESTATE;
   cudaError_t e = cudaStreamSynchronize(h->stream);
   if (e == cudaSuccess)
-    e = rows_to_device(h, state_in, 0, h->g.d);
+    e = rows_to_device(h, set_of_step(h, k - 1), state_in, 0, h->g.d);
   if (e == cudaSuccess) e = cudaMemsetAsync(keys(h), 0, 2 * sizeof(u64), h->stream);
   if (e != cudaSuccess) return sticky(h, e);
-  pf::StepParams p = base_params(h, k, pf::MODE_SAMPLE);
-  host_inputs(h, p, z_k, u_km1);
-  pf_status s = launch(h, p);
+  pf_status s;
+  if (h->g.central) {
+    pf::CentralParams c = central_params(h, k);
+    c.first = 1;   // sample + weight only (a1-a3)
+    host_inputs(h, c, z_k, u_km1);
+    s = launch_central(h, c);
+  } else {
+    pf::StepParams p = base_params(h, k, pf::MODE_SAMPLE);
+    host_inputs(h, p, z_k, u_km1);
+    s = launch(h, p);
+  }
   if (s != PF_OK) return s;
   h->step = k;
   e = cudaStreamSynchronize(h->stream);
   if (e == cudaSuccess)
-    e = rows_to_host(h, state_out, 0, h->g.d);
-  if (e == cudaSuccess) e = rows_to_host(h, logw_out, h->g.d, 1);
+    e = rows_to_host(h, set_of_step(h, k), state_out, 0, h->g.d);
+  if (e == cudaSuccess) e = rows_to_host(h, set_of_step(h, k), logw_out, h->g.d, 1);
   return sticky(h, e);
 }
 
@@ -594,6 +708,7 @@ pf_status pf_debug_resample(pf_handle* h, const uint32_t* q, const uint32_t* ua,
                             int32_t* ancestors, uint64_t* prob, int32_t* alias) {
   if (!h || !q || !ua || !ub || !ancestors) return PF_EINVAL;
   if (h->err != PF_OK) return h->err;
+  if (h->g.central) return PF_ESTATE;
   const long long n = h->g.N * h->g.m;
   DevBuf<uint32_t> dq, dua, dub;
   DevBuf<int> danc, dal;
@@ -622,12 +737,12 @@ pf_status pf_debug_resample(pf_handle* h, const uint32_t* q, const uint32_t* ua,
 pf_status pf_debug_exchange(pf_handle* h, const float* logw, int64_t* src) {
   if (!h || !logw || !src) return PF_EINVAL;
   if (h->err != PF_OK) return h->err;
-  if (h->cfg.world != 1) return PF_ESTATE;
+  if (h->cfg.world != 1 || h->g.central) return PF_ESTATE;
   const long long M = h->g.M_local;
   DevBuf<long long> dsrc;
   cudaError_t e = dsrc.alloc(M);
   if (e == cudaSuccess) e = cudaStreamSynchronize(h->stream);
-  if (e == cudaSuccess) e = rows_to_device(h, logw, h->g.d, 1);
+  if (e == cudaSuccess) e = rows_to_device(h, h->parts, logw, h->g.d, 1);
   if (e != cudaSuccess) return sticky(h, e);
   const long long s = h->step > 0 ? h->step : 1;
   pf_status st = publish(h, s);
@@ -644,6 +759,7 @@ pf_status pf_debug_exchange(pf_handle* h, const float* logw, int64_t* src) {
 
 pf_status pf_set_trace(pf_handle* h, int32_t enable) {
   if (!h) return PF_EINVAL;
+  if (h->g.central) return enable ? PF_ESTATE : PF_OK;
   if (enable && !h->trace) {
     cudaError_t e = cudaStreamSynchronize(h->stream);
     if (e == cudaSuccess) e = cudaMalloc(&h->d_src, sizeof(long long) * h->g.M_local);
@@ -717,21 +833,21 @@ int32_t pf_supported(int32_t* n_joints, int32_t* m, int32_t cap) {
 }  // extern "C"
 
 namespace {
-cudaError_t rows_to_device(pf_handle* h, const float* host, int row0, int nrows) {
+cudaError_t rows_to_device(pf_handle* h, float* base, const float* host, int row0, int nrows) {
   const size_t m = h->g.m;
   for (int r = 0; r < nrows; ++r) {
-    cudaError_t e = cudaMemcpy2D(h->parts + (row0 + r) * m, sizeof(float) * h->g.ROW,
+    cudaError_t e = cudaMemcpy2D(base + (row0 + r) * m, sizeof(float) * h->g.ROW,
                                  host + static_cast<size_t>(r) * h->g.M_local, sizeof(float) * m, sizeof(float) * m,
                                  h->g.n_local, cudaMemcpyHostToDevice);
     if (e != cudaSuccess) return e;
   }
   return cudaSuccess;
 }
-cudaError_t rows_to_host(pf_handle* h, float* host, int row0, int nrows) {
+cudaError_t rows_to_host(pf_handle* h, const float* base, float* host, int row0, int nrows) {
   const size_t m = h->g.m;
   for (int r = 0; r < nrows; ++r) {
     cudaError_t e = cudaMemcpy2D(host + static_cast<size_t>(r) * h->g.M_local, sizeof(float) * m,
-                                 h->parts + (row0 + r) * m, sizeof(float) * h->g.ROW, sizeof(float) * m,
+                                 base + (row0 + r) * m, sizeof(float) * h->g.ROW, sizeof(float) * m,
                                  h->g.n_local, cudaMemcpyDeviceToHost);
     if (e != cudaSuccess) return e;
   }

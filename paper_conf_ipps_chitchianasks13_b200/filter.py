@@ -49,6 +49,10 @@ class ParticleFilter:
     ``n_filters`` (global N), exchange scheme ``topo`` and ``t`` particles per
     exchange; ``resampler`` 'rws' | 'vose'.  ``rank``/``world`` select this
     process's shard of the sub-filters (pf.h).
+
+    ``n_filters=1`` with ``m > 1024`` (a multiple of 4096) is the paper's
+    centralized filter (§VI, Fig. 9): one filter resampled
+    globally over all ``m`` particles (RWS; pf_central.cu).
     """
 
     def __init__(self, mu0, sigma0, model: ArmModel | None = None, m: int = 256, n_filters: int = 4096,
@@ -76,14 +80,18 @@ class ParticleFilter:
             self.h = B.pf_init(self.cfg, mc, bufs, self.stream.cuda_stream, _f32(mu0), _f32(sigma0))
         self.shard = B.pf_get_shard(self.h)
         self.M_local = self.shard.n_local * m
+        self.central = n_filters == 1 and m > 1024
+        self._k = 0
         self._xhat = np.zeros(self.d, np.float32)
 
     # -- views of the caller-owned buffers (torch, device) -------------------
     @property
     def particles(self) -> torch.Tensor:
-        """Device particle blocks [n_local][d+1][m] (rows 0..d-1 state, row d log-weight)."""
+        """Device particle blocks [n_local][d+1][m] (rows 0..d-1 state, row d log-weight).
+        Centralized filter: the buffer holding the current step's set (ping-pong, k & 1)."""
         n = self.shard.n_local * (self.d + 1) * self.m
-        return self._parts[: 4 * n].view(torch.float32).view(self.shard.n_local, self.d + 1, self.m)
+        off = 4 * n * (self._k & 1) if self.central else 0
+        return self._parts[off: off + 4 * n].view(torch.float32).view(self.shard.n_local, self.d + 1, self.m)
 
     @property
     def mailbox(self) -> torch.Tensor:
@@ -104,11 +112,13 @@ class ParticleFilter:
             B.pf_step(self.h, z.data_ptr(), u.data_ptr())
         else:
             B.pf_step(self.h, _f32(z), _f32(u))
+        self._k += 1
 
     def step_batch(self, zs: torch.Tensor, us: torch.Tensor, est: torch.Tensor | None = None) -> None:
         """T steps with device-resident inputs zs [T][nj+2], us [T][nj]; est [T][4+d]."""
         assert zs.is_cuda and us.is_cuda and zs.dtype == torch.float32 and us.dtype == torch.float32
         B.pf_step_batch(self.h, zs.shape[0], zs.data_ptr(), us.data_ptr(), None if est is None else est.data_ptr())
+        self._k += zs.shape[0]
 
     def estimate(self):
         """(x_hat [d], logw, global index) of the particle with the highest weight."""
@@ -126,16 +136,19 @@ class ParticleFilter:
         s = np.zeros((self.d, self.M_local), np.float32)
         w = np.zeros(self.M_local, np.float32)
         k = B.pf_get_particles(self.h, s, w)
+        self._k = k
         return s, w, k
 
     def set_particles(self, state, logw, step: int) -> None:
         B.pf_set_particles(self.h, _f32(state), _f32(logw), step)
+        self._k = step
 
     # -- test hooks ----------------------------------------------------------
     def debug_sample_weight(self, state_in, z, u, k: int):
         s_out = np.zeros((self.d, self.M_local), np.float32)
         w_out = np.zeros(self.M_local, np.float32)
         B.pf_debug_sample_weight(self.h, _f32(state_in), _f32(z), _f32(u), k, s_out, w_out)
+        self._k = k
         return s_out, w_out
 
     def debug_resample(self, q, ua, ub):

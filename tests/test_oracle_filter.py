@@ -133,3 +133,21 @@ def test_step_subset_equals_whole_filter(orc, W):
         for i, n in enumerate(subs):
             np.testing.assert_array_equal(os_[:, i * 32:(i + 1) * 32], s1[:, n * 32:(n + 1) * 32])
             np.testing.assert_array_equal(ow[i * 32:(i + 1) * 32], w1[n * 32:(n + 1) * 32])
+
+
+def test_central_slots_equals_whole_filter(orc, W):
+    # the slot-sampled centralized oracle reproduces the whole-filter step
+    for res in ("rws", "vose"):
+        cfg = orc.Config(m=2048, n_filters=1, t=0, topo="none", resampler=res, seed=21)
+        md = orc.Model(n_joints=5)
+        tr = W.make_trajectory(5, 10, 0)
+        f = orc.Filter(cfg, md, tr["mu0"], tr["sigma0"])
+        s0 = W.random_particles(tr, 2048, 4)
+        w0 = W.random_logw(1, 2048, 4).ravel()
+        f.set(s0, w0, 2)
+        f.step(tr["Z"][3], tr["U"][2])
+        s1, w1, _ = f.get()
+        slots = [0, 1, 777, 2047]
+        os_, ow = orc.central_slots(cfg, md, s0, w0, 3, tr["Z"][3], tr["U"][2], slots)
+        np.testing.assert_array_equal(os_, s1[:, slots])
+        np.testing.assert_array_equal(ow, w1[slots])
