@@ -11,7 +11,7 @@ import ctypes as C
 import os
 
 HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(HERE, "libpf_b200.so")
+LIB_PATH = os.environ.get("PF_LIB") or os.path.join(HERE, "libpf_b200.so")   # PF_LIB: dev A/B builds
 
 PF_OK, PF_EINVAL, PF_ENOMEM, PF_ECUDA, PF_ESTATE, PF_EUNSUPPORTED = 0, -1, -2, -3, -5, -6
 PF_TOPO_NONE, PF_TOPO_RING, PF_TOPO_TORUS2D, PF_TOPO_ALL2ALL = 0, 1, 2, 3
@@ -222,10 +222,11 @@ def pf_supported() -> list[tuple[int, int]]:
     return list(zip(list(nj), list(m)))
 
 
-def pf_debug_math(fn: str, words, n: int):
-    """Evaluate a contract function on the device; words: uint32 numpy array."""
+def pf_debug_math(fn: str, words, n: int, x2: bool = False):
+    """Evaluate a contract function on the device; words: uint32 numpy array.
+    x2: through the packed f32x2 code path (element pairs; n even)."""
     import numpy as np
-    k = PF_MATH[fn]
+    k = PF_MATH[fn] | (0x100 if x2 else 0)
     w = np.ascontiguousarray(words, dtype=np.uint32)
     out_n = 2 * n if fn in ("sincos2pi", "normal_pair") else 4 * n if fn == "philox" else n
     out = np.zeros(max(out_n, 1), np.uint32)

@@ -130,13 +130,12 @@ __global__ void __launch_bounds__(256) cz_step(const CentralParams C) {
     }
     const float* xa = C.in + a;
     auto x = [xa, M](int c) { return __ldg(xa + c * M); };
-    float xo[D];
     NoiseGen gen{p, C.k, C.rk, u32x4{0u, 0u, b0.z, b0.w}};
-    SamplePairs<NJ, 0>::run(C.mc, hsu_s, x, gen, xo);
-    const float l = arm_loglik<NJ>(C.mc, z_s, xo);
-#pragma unroll
-    for (int c = 0; c < D; ++c) C.out[c * M + i] = xo[c];
-    C.out[D * M + i] = l;
+    ArmAcc A;
+    float* out = C.out + i;
+    SampleStream<NJ, 0>::run(C.mc, hsu_s, z_s, x, gen, A, [out, M](int c, float v) { out[c * M] = v; });
+    const float l = arm_finish(C.mc, z_s, A);
+    out[D * M] = l;
     const u64 key = order_key(l, p);
     best = key > best ? key : best;
   }

@@ -41,6 +41,38 @@ __global__ void math_kernel(int fn, const uint32_t* in, uint32_t* out, long long
   }
 }
 
+// The packed (f32x2) evaluation of the same functions on element pairs
+// (2i, 2i+1); n even.
+__global__ void math_x2_kernel(int fn, const uint32_t* in, uint32_t* out, long long n) {
+  for (long long i = blockIdx.x * static_cast<long long>(blockDim.x) + threadIdx.x; 2 * i < n;
+       i += static_cast<long long>(gridDim.x) * blockDim.x) {
+    const uint32_t a = in[2 * i], b = in[2 * i + 1];
+    const pf::f2 x = pf::pk(__uint_as_float(a), __uint_as_float(b));
+    pf::f2 s, c;
+    switch (fn) {
+      case PF_MATH_SIN: pf::sincos_c2(x, s, c); out[2 * i] = __float_as_uint(pf::lo2(s));
+        out[2 * i + 1] = __float_as_uint(pf::hi2(s)); break;
+      case PF_MATH_COS: pf::sincos_c2(x, s, c); out[2 * i] = __float_as_uint(pf::lo2(c));
+        out[2 * i + 1] = __float_as_uint(pf::hi2(c)); break;
+      case PF_MATH_LOG: s = pf::log_c2(x); out[2 * i] = __float_as_uint(pf::lo2(s));
+        out[2 * i + 1] = __float_as_uint(pf::hi2(s)); break;
+      case PF_MATH_SQRT: s = pf::sqrt_pos2(x, pf::pk(-__uint_as_float(a), -__uint_as_float(b)));
+        out[2 * i] = __float_as_uint(pf::lo2(s)); out[2 * i + 1] = __float_as_uint(pf::hi2(s)); break;
+      case PF_MATH_SINCOS2PI: pf::sincos2pi_c2(a, b, s, c);
+        out[4 * i] = __float_as_uint(pf::lo2(s)); out[4 * i + 1] = __float_as_uint(pf::lo2(c));
+        out[4 * i + 2] = __float_as_uint(pf::hi2(s)); out[4 * i + 3] = __float_as_uint(pf::hi2(c)); break;
+      case PF_MATH_NORMAL_PAIR: {
+        pf::f2 z0, z1;
+        pf::normal_pair2(a, in[n + 2 * i], b, in[n + 2 * i + 1], z0, z1);
+        out[4 * i] = __float_as_uint(pf::lo2(z0)); out[4 * i + 1] = __float_as_uint(pf::lo2(z1));
+        out[4 * i + 2] = __float_as_uint(pf::hi2(z0)); out[4 * i + 3] = __float_as_uint(pf::hi2(z1));
+        break;
+      }
+      default: break;
+    }
+  }
+}
+
 __global__ void sqrt_check_kernel(uint32_t lo, uint32_t hi, unsigned long long* bad) {
   unsigned long long local = 0;
   for (unsigned long long b = lo + blockIdx.x * static_cast<unsigned long long>(blockDim.x) + threadIdx.x; b <= hi;
@@ -55,8 +87,11 @@ __global__ void sqrt_check_kernel(uint32_t lo, uint32_t hi, unsigned long long* 
 
 extern "C" {
 
-pf_status pf_debug_math(int32_t fn, const uint32_t* in, uint32_t* out, int64_t n) {
+pf_status pf_debug_math(int32_t fn_flags, const uint32_t* in, uint32_t* out, int64_t n) {
+  const bool x2 = (fn_flags & PF_MATH_X2) != 0;
+  const int32_t fn = fn_flags & ~PF_MATH_X2;
   if (!in || !out || n < 0 || fn < PF_MATH_SIN || fn > PF_MATH_PHILOX) return PF_EINVAL;
+  if (x2 && ((n & 1) || fn == PF_MATH_EXPQ || fn == PF_MATH_PHILOX)) return PF_EINVAL;
   const long long in_words = fn == PF_MATH_NORMAL_PAIR ? 2 * n : fn == PF_MATH_PHILOX ? 4 * n + 2 : n;
   const long long out_words = (fn == PF_MATH_SINCOS2PI || fn == PF_MATH_NORMAL_PAIR) ? 2 * n
                               : fn == PF_MATH_PHILOX                                  ? 4 * n
@@ -66,7 +101,12 @@ pf_status pf_debug_math(int32_t fn, const uint32_t* in, uint32_t* out, int64_t n
   if (e == cudaSuccess) e = cudaMalloc(&dout, 4 * (out_words ? out_words : 1));
   if (e == cudaSuccess) e = cudaMemcpy(din, in, 4 * in_words, cudaMemcpyHostToDevice);
   if (e == cudaSuccess && n > 0) {
-    math_kernel<<<static_cast<int>((n + 255) / 256 < 4096 ? (n + 255) / 256 : 4096), 256>>>(fn, din, dout, n);
+    const int grid = static_cast<int>((n + 255) / 256 < 4096 ? (n + 255) / 256 : 4096);
+    if (x2) {
+      math_x2_kernel<<<grid, 256>>>(fn, din, dout, n);
+    } else {
+      math_kernel<<<grid, 256>>>(fn, din, dout, n);
+    }
     e = cudaGetLastError();
   }
   if (e == cudaSuccess) e = cudaMemcpy(out, dout, 4 * out_words, cudaMemcpyDeviceToHost);

@@ -5,14 +5,17 @@
 #include "pf_registry.h"
 
 namespace pf {
-#define PF_LARGE_D_ENTRIES(NJ, RES)                                                                \
+#define PF_LARGE_D_ENTRIES(NJ, RES, GW256, MINB256)                                                \
   PF_ENTRY(NJ, 32, RES, 1, 4, 1, 1, 1), PF_ENTRY(NJ, 64, RES, 2, 2, 1, 1, 1),                       \
-      PF_ENTRY(NJ, 128, RES, 4, 1, 1, 1, 1), PF_ENTRY(NJ, 256, RES, 8, 1, 1, 1, 4),                 \
+      PF_ENTRY(NJ, 128, RES, 4, 1, 1, 1, 1), PF_ENTRY(NJ, 256, RES, GW256, 1, 1, 1, MINB256),       \
       PF_ENTRY(NJ, 512, RES, 16, 1, 1, 1, 1), PF_ENTRY(NJ, 1024, RES, 16, 1, 1, 1, 1)
 const KernelEntry kEntriesNJ28[] = {
-    PF_LARGE_D_ENTRIES(28, 0), PF_LARGE_D_ENTRIES(28, 1),
+    // m = 256 (config C4), measured: RWS two particles per thread (packed f32x2 path), Vose one
+    PF_LARGE_D_ENTRIES(28, 0, 4, 6), PF_LARGE_D_ENTRIES(28, 1, 8, 4),
+    PF_ENTRY(28, 256, 0, 8, 1, 1, 1, 4),
     PF_ENTRY(28, 256, 0, 8, 1, 1, 1, 3), PF_ENTRY(28, 256, 0, 4, 1, 1, 1, 4), PF_ENTRY(28, 256, 0, 8, 1, 2, 1, 3),
     PF_ENTRY(28, 256, 1, 8, 1, 1, 1, 3), PF_ENTRY(28, 256, 1, 4, 1, 1, 1, 4),
+    PF_ENTRY(28, 256, 1, 4, 1, 1, 1, 6),
 };
 const int kNumEntriesNJ28 = sizeof(kEntriesNJ28) / sizeof(kEntriesNJ28[0]);
 }  // namespace pf

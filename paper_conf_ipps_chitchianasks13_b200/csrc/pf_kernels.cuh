@@ -44,6 +44,7 @@ enum : int { RES_RWS = 0, RES_VOSE = 1 };
 
 struct StepParams {
   ArmConsts mc;
+  ArmConsts2 mc2;          // mc with every field duplicated (packed f32x2 operands)
   float* parts;            // [n_local][D+1][M] blocked SoA (row D = log-weight)
   const float* mb_prev;    // mailbox parity (k-1)&1 : [n_ext][tt][E]
   float* mb_cur;           // mailbox parity k&1
@@ -113,7 +114,11 @@ __device__ __forceinline__ void mbar_wait(u64* bar, uint32_t parity) {
 // group; the per-particle sample/weight loop over a thread's P slots is
 // unrolled UNR times (P for full unrolling; 1 keeps one copy of the
 // ~10–40 KB per-particle code in the instruction cache).
-template <int NJ_, int M_, int RES_, int GW_, int S_, int NSTAGE_, int UNR_, int MINB_, int EARLY_ = 0>
+#ifndef PF_X2_DEFAULT
+#define PF_X2_DEFAULT 1
+#endif
+template <int NJ_, int M_, int RES_, int GW_, int S_, int NSTAGE_, int UNR_, int MINB_, int EARLY_ = 0,
+          int X2_ = PF_X2_DEFAULT>
 struct KCfg {
   static constexpr int EARLY = EARLY_;       // start the next TMA load right after the sample loop
   static constexpr int NJ = NJ_, M = M_, RES = RES_, GW = GW_, S = S_, NSTAGE = NSTAGE_, UNR = UNR_;
@@ -125,6 +130,7 @@ struct KCfg {
   static constexpr int ROW = (D + 1) * M;    // floats per sub-filter block
   static constexpr bool SCAN32 = (M <= 512);  // Q <= M 2^22 fits 32 bits
   static constexpr bool STAGED = UNR < P;    // rolled sample loop: per-slot values via smem
+  static constexpr bool X2 = X2_ && (P % 2 == 0);   // sample two particles at once (packed f32x2)
   static_assert(P >= 1 && P * T == M, "M must be a multiple of the group size");
   static_assert(P <= 32, "exclusion masks are 32-bit");
   static_assert(S >= 1 && S <= 15, "named barriers 1..S");
@@ -144,7 +150,8 @@ struct KCfg {
   static constexpr size_t group_bytes = (g_bar + 32 + 127) / 128 * 128;
   // per-CTA
   static constexpr size_t c_zin = 0;          // float [64]: z (NJ+2), h_s u (NJ)
-  static constexpr size_t c_groups = 256;
+  static constexpr size_t c_zin2 = 256;       // f2 [64]: the same, each value duplicated (packed operands)
+  static constexpr size_t c_groups = 768;
   static constexpr size_t smem = c_groups + S * group_bytes;
   // slot j of group thread t: strided, so chunk j of the group covers the
   // contiguous slots [jT, (j+1)T) and every row store is coalesced
@@ -442,17 +449,51 @@ struct NoiseGen {
   }
 };
 
+// Streamed sample + weight of one particle (F8–F10), Box–Muller pair by
+// pair; out(c, v) stores component c of the new state.
 template <int NJ, int QP>
-struct SamplePairs {
+struct SampleStream {
   static constexpr int D = NJ + 4;
-  template <typename X>
-  __device__ __forceinline__ static void run(const ArmConsts& mc, const float* hsu, const X& x, NoiseGen& gen,
-                                             float (&xo)[NJ + 4]) {
+  template <typename X, typename O>
+  __device__ __forceinline__ static void run(const ArmConsts& mc, const float* hsu, const float* z, const X& x,
+                                             NoiseGen& gen, ArmAcc& A, const O& out) {
     float z0, z1;
     gen.template pair<QP>(z0, z1);
-    xo[2 * QP] = arm_sample_comp<NJ, 2 * QP>(mc, hsu, x, z0);
-    if constexpr (2 * QP + 1 < D) xo[2 * QP + 1] = arm_sample_comp<NJ, 2 * QP + 1>(mc, hsu, x, z1);
-    if constexpr (QP + 1 < (D + 1) / 2) SamplePairs<NJ, QP + 1>::run(mc, hsu, x, gen, xo);
+    out(2 * QP, arm_sample_take<NJ, 2 * QP>(mc, hsu, z, x, z0, A));
+    if constexpr (2 * QP + 1 < D) out(2 * QP + 1, arm_sample_take<NJ, 2 * QP + 1>(mc, hsu, z, x, z1, A));
+    if constexpr (QP + 1 < (D + 1) / 2) SampleStream<NJ, QP + 1>::run(mc, hsu, z, x, gen, A, out);
+  }
+};
+
+// Two particles A, B at once: the same Philox words per particle, the
+// Box–Muller arithmetic packed (normal_pair2).
+struct NoiseGen2 {
+  uint32_t pa, pb, k;
+  const uint32_t (&rk)[20];
+  u32x4 ba, bb;
+  template <int QP>
+  __device__ __forceinline__ void pair(f2& z0, f2& z1) {
+    constexpr int w = 2 + 2 * QP;
+    if constexpr ((w & 3) == 0) {
+      ba = philox4x32_10_rk(pa, k, 0u, static_cast<uint32_t>(w >> 2), rk);
+      bb = philox4x32_10_rk(pb, k, 0u, static_cast<uint32_t>(w >> 2), rk);
+    }
+    normal_pair2((w & 3) == 2 ? ba.z : ba.x, (w & 3) == 2 ? ba.w : ba.y, (w & 3) == 2 ? bb.z : bb.x,
+                 (w & 3) == 2 ? bb.w : bb.y, z0, z1);
+  }
+};
+
+template <int NJ, int QP>
+struct SampleStream2 {
+  static constexpr int D = NJ + 4;
+  template <typename X, typename O>
+  __device__ __forceinline__ static void run(const ArmConsts2& mc, const f2* hsu2, const f2* z2, const X& x,
+                                             NoiseGen2& gen, ArmAcc2& A, const O& out) {
+    f2 z0, z1;
+    gen.template pair<QP>(z0, z1);
+    out(2 * QP, arm_sample_take2<NJ, 2 * QP>(mc, hsu2, z2, x, z0, A));
+    if constexpr (2 * QP + 1 < D) out(2 * QP + 1, arm_sample_take2<NJ, 2 * QP + 1>(mc, hsu2, z2, x, z1, A));
+    if constexpr (QP + 1 < (D + 1) / 2) SampleStream2<NJ, QP + 1>::run(mc, hsu2, z2, x, gen, A, out);
   }
 };
 
@@ -502,6 +543,8 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
   extern __shared__ __align__(128) unsigned char smem[];
   float* z_s = reinterpret_cast<float*>(smem + C::c_zin);
   float* hsu_s = z_s + NJ + 2;
+  f2* z2_s = reinterpret_cast<f2*>(smem + C::c_zin2);
+  f2* hsu2_s = z2_s + NJ + 2;
 
   const int g = threadIdx.x / C::T;
   unsigned char* gs = smem + C::c_groups + g * C::group_bytes;
@@ -564,8 +607,16 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
     if (gid0 < P.n_local) pending = atomicAdd(P.work, 1u);
   }
   if (do_sample) {
-    if (threadIdx.x < NJ + 2) z_s[threadIdx.x] = P.z ? P.z[threadIdx.x] : P.zin[threadIdx.x];
-    if (threadIdx.x < NJ) hsu_s[threadIdx.x] = P.mc.hs * (P.u ? P.u[threadIdx.x] : P.uin[threadIdx.x]);
+    if (threadIdx.x < NJ + 2) {
+      const float v = P.z ? P.z[threadIdx.x] : P.zin[threadIdx.x];
+      z_s[threadIdx.x] = v;
+      z2_s[threadIdx.x] = bc(v);
+    }
+    if (threadIdx.x < NJ) {
+      const float v = P.mc.hs * (P.u ? P.u[threadIdx.x] : P.uin[threadIdx.x]);
+      hsu_s[threadIdx.x] = v;
+      hsu2_s[threadIdx.x] = bc(v);
+    }
   }
   __syncthreads();
 
@@ -780,7 +831,50 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
       }
     }
 
-    if (do_sample) {
+    if (C::X2 && do_sample) {
+      // ---- a9 gather (smem) + a1 RNG + a2 sample + a3 weight + a10 store,
+      //      two particles (slots j, j+1 of this thread) at a time with the
+      //      floating-point work packed (f32x2, bit-identical lane by lane)
+#pragma unroll(C::UNR > 1 ? C::UNR / 2 : 1)
+      for (int j = 0; j < PP; j += 2) {
+        const int sa = C::slot(G.t, j), sb = C::slot(G.t, j + 1);
+        int a0, a1;
+        uint32_t za2, za3, zb2, zb3;
+        if constexpr (C::STAGED) {
+          a0 = reinterpret_cast<const int*>(ws)[sa];
+          a1 = reinterpret_cast<const int*>(ws)[sb];
+          const uint2 pa = bzw_s[sa], pb = bzw_s[sb];
+          za2 = pa.x;
+          za3 = pa.y;
+          zb2 = pb.x;
+          zb3 = pb.y;
+        } else {
+          a0 = anc[j];
+          a1 = anc[j + 1];
+          za2 = bz[j];
+          za3 = bw[j];
+          zb2 = bz[j + 1];
+          zb3 = bw[j + 1];
+        }
+        const float* xa = xs + a0;
+        const float* xb = xs + a1;
+        auto x = [xa, xb](int c) { return pk(xa[c * M], xb[c * M]); };
+        float* outa = gblk + sa;
+        float* outb = gblk + sb;
+        NoiseGen2 gen{pbase + static_cast<uint32_t>(sa), pbase + static_cast<uint32_t>(sb), P.k, P.rk,
+                      u32x4{0u, 0u, za2, za3}, u32x4{0u, 0u, zb2, zb3}};
+        ArmAcc2 A;
+        SampleStream2<NJ, 0>::run(P.mc2, hsu2_s, z2_s, x, gen, A, [outa, outb](int c, f2 v) {
+          outa[c * M] = lo2(v);
+          outb[c * M] = hi2(v);
+        });
+        const f2 l = arm_finish2(P.mc2, z2_s, A);
+        outa[D * M] = lo2(l);
+        outb[D * M] = hi2(l);
+        reinterpret_cast<float*>(bzw_s)[2 * sa] = lo2(l);   // own slots, after their Philox words were read
+        reinterpret_cast<float*>(bzw_s)[2 * sb] = hi2(l);
+      }
+    } else if (do_sample) {
       // ---- a9 gather (smem) + a1 RNG + a2 sample + a3 weight + a10 store,
       //      one particle at a time (coalesced rows: consecutive threads,
       //      consecutive slots)
@@ -801,13 +895,11 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
         }
         const float* xa = xs + a;
         auto x = [xa](int c) { return xa[c * M]; };
-        float xo[D];
-        NoiseGen gen{pbase + static_cast<uint32_t>(s), P.k, P.rk, u32x4{0u, 0u, z2, z3}};
-        SamplePairs<NJ, 0>::run(P.mc, hsu_s, x, gen, xo);
-        const float l = arm_loglik<NJ>(P.mc, z_s, xo);
         float* out = gblk + s;
-#pragma unroll
-        for (int c = 0; c < D; ++c) out[c * M] = xo[c];
+        NoiseGen gen{pbase + static_cast<uint32_t>(s), P.k, P.rk, u32x4{0u, 0u, z2, z3}};
+        ArmAcc A;
+        SampleStream<NJ, 0>::run(P.mc, hsu_s, z_s, x, gen, A, [out](int c, float v) { out[c * M] = v; });
+        const float l = arm_finish(P.mc, z_s, A);
         out[D * M] = l;
         reinterpret_cast<float*>(bzw_s)[2 * s] = l;   // own slot, after its Philox words were read
 

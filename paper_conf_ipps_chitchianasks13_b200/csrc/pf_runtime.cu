@@ -212,6 +212,13 @@ pf::StepParams base_params(pf_handle* h, long long k, int mode) {
   pf::StepParams p;
   std::memset(&p, 0, sizeof(p));
   p.mc = h->mc;
+  auto dup = [](float v) {
+    uint32_t b;
+    std::memcpy(&b, &v, 4);
+    return (static_cast<unsigned long long>(b) << 32) | b;
+  };
+  p.mc2 = {dup(h->mc.lj), dup(h->mc.hs), dup(h->mc.s_th), dup(h->mc.s_pos), dup(h->mc.s_vel), dup(h->mc.inv_cam),
+           dup(h->mc.inv_thm)};
   p.parts = h->parts;
   p.mb_prev = mailbox_parity(h, k - 1);
   p.mb_cur = mailbox_parity(h, k);

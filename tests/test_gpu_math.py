@@ -27,21 +27,23 @@ def test_sqrt_exhaustive_on_box_muller_domain(B):
     assert B.pf_debug_check_sqrt(lo, hi) == 0
 
 
+@pytest.mark.parametrize("x2", [False, True], ids=["scalar", "packed"])
 @pytest.mark.parametrize("fn", ["sin", "cos"])
-def test_sincos_bit_exact(B, orc, fn):
+def test_sincos_bit_exact(B, orc, fn, x2):
     rng = np.random.default_rng(1)
     x = np.concatenate([rng.uniform(-4, 4, 3000), rng.uniform(-60, 60, 3000), [0.0, -0.0, 0.7853981, 1e-30]])
     x = x.astype(np.float32)
-    got = B.pf_debug_math(fn, _f32bits(x), len(x)).view(np.float32)
+    got = B.pf_debug_math(fn, _f32bits(x), len(x), x2).view(np.float32)
     ref = np.array([orc.s_sin(float(v)) if fn == "sin" else orc.s_cos(float(v)) for v in x], np.float32)
     np.testing.assert_array_equal(got.view(np.uint32), ref.view(np.uint32))
 
 
-def test_log_bit_exact(B, orc):
+@pytest.mark.parametrize("x2", [False, True], ids=["scalar", "packed"])
+def test_log_bit_exact(B, orc, x2):
     rng = np.random.default_rng(2)
     n1 = np.concatenate([rng.integers(1, 1 << 24, 5000) | 1, [1, (1 << 24) - 1]])
     u = (n1.astype(np.float64) * 2.0**-24).astype(np.float32)
-    got = B.pf_debug_math("log", _f32bits(u), len(u)).view(np.float32)
+    got = B.pf_debug_math("log", _f32bits(u), len(u), x2).view(np.float32)
     ref = np.array([orc.s_log(float(v)) for v in u], np.float32)
     np.testing.assert_array_equal(got.view(np.uint32), ref.view(np.uint32))
 
@@ -54,17 +56,19 @@ def test_expq_bit_exact(B, orc):
     np.testing.assert_array_equal(got, ref)
 
 
-def test_normal_pair_and_sincos2pi_bit_exact(B, orc):
+@pytest.mark.parametrize("x2", [False, True], ids=["scalar", "packed"])
+def test_normal_pair_and_sincos2pi_bit_exact(B, orc, x2):
     rng = np.random.default_rng(4)
     n = 4000
     x0 = rng.integers(0, 2**32, n, dtype=np.uint64).astype(np.uint32)
     x1 = rng.integers(0, 2**32, n, dtype=np.uint64).astype(np.uint32)
     x0[:4] = [0, 0xFFFFFFFF, 0x1FF, 0x200]
-    got = B.pf_debug_math("normal_pair", np.concatenate([x0, x1]), n).view(np.float32).reshape(n, 2)
+    x1[4:8] = [0, 1 << 29, 2 << 29, 3 << 29]   # exact quadrant multiples: f = 0, signed zeros
+    got = B.pf_debug_math("normal_pair", np.concatenate([x0, x1]), n, x2).view(np.float32).reshape(n, 2)
     ref = np.array([orc.s_normal_pair(int(a), int(b)) for a, b in zip(x0, x1)], np.float32)
     np.testing.assert_array_equal(got.view(np.uint32), ref.view(np.uint32))
     m = (x1 >> 9).astype(np.uint32)
-    got2 = B.pf_debug_math("sincos2pi", m, n).view(np.float32).reshape(n, 2)
+    got2 = B.pf_debug_math("sincos2pi", m, n, x2).view(np.float32).reshape(n, 2)
     ref2 = np.array([orc.s_sincos2pi(int(v)) for v in m], np.float32)
     np.testing.assert_array_equal(got2.view(np.uint32), ref2.view(np.uint32))
 
@@ -78,3 +82,12 @@ def test_philox_kat_on_device(B, orc):
         words = np.array([r[0], r[1], r[2], r[3], r[4], r[5]], np.uint32)
         out = B.pf_debug_math("philox", words, 1)
         assert list(map(int, out)) == r[6:10]
+
+
+def test_sqrt_packed_matches_scalar(B):
+    rng = np.random.default_rng(5)
+    x = np.concatenate([rng.uniform(1.2e-7, 33.3, 4000), [1.1920929e-07, 33.27]]).astype(np.float32)
+    a = B.pf_debug_math("sqrt", _f32bits(x), len(x))
+    b = B.pf_debug_math("sqrt", _f32bits(x), len(x), True)
+    np.testing.assert_array_equal(a, b)
+    np.testing.assert_array_equal(a.view(np.float32), np.sqrt(x))
