@@ -79,7 +79,9 @@ typedef struct {
  * sub-filters [r N/W, (r+1) N/W); torus — rank r owns rows
  * [r R/W, (r+1) R/W) of the R x C grid. */
 typedef struct {
-  int32_t m;                /* particles per sub-filter, power of two in [32, 1024]  */
+  int32_t m;                /* particles per sub-filter, power of two in [32, 1024]; */
+                            /* n_filters == 1 and m > 1024: the centralized filter  */
+                            /* (multiple of 4096, <= 2^26; Vose <= 2^20), see below */
   int64_t n_filters;        /* N, GLOBAL number of sub-filters                       */
   int32_t t;                /* particles per exchange per neighbour; deg*t < m (R19) */
   int32_t topo;             /* pf_topology                                           */
@@ -141,7 +143,12 @@ pf_status pf_query_sizes(const pf_config* cfg, const pf_model_params* model, pf_
  * cudaStream_t (NULL = legacy default stream).  Validation (PF_EINVAL): m a
  * power of two in [32, 1024]; deg*t < m; N % world == 0 (ring) or
  * R % world == 0 and R*C == N (torus); N*m per shard <= 2^31; global N*m <= 2^32;
- * 0 <= rank < world; unsupported n_joints -> PF_EUNSUPPORTED. */
+ * 0 <= rank < world; unsupported n_joints -> PF_EUNSUPPORTED.
+ * Centralized filter ("a sequential, centralized particle filter", PAPER.md:18
+ * §VI; Fig. 5 and 9): n_filters == 1 and m > 1024 resamples
+ * all m particles globally (RWS or Vose over every slot, no exchange:
+ * topo NONE or t == 0; world == 1); m a multiple of 4096 and <= 2^26, Vose
+ * m <= 2^20 (PF_EUNSUPPORTED above: its u64 alias sums reach m^2 2^22). */
 pf_status pf_init(const pf_config* cfg, const pf_model_params* model, const pf_buffers* buffers,
                   void* cuda_stream, const float* mu0, const float* sigma0, pf_handle** out);
 
@@ -211,7 +218,8 @@ pf_status pf_debug_sample_weight(pf_handle* h, const float* state_in, const floa
 /* Resampling (a8) of integer weights q [N][m] (host, each row with
  * sum > 0 and sum <= 2^32) with explicit uniforms ua, ub [N][m] (host):
  * ancestors [N][m] (host).  Vose only: prob [N][m] (uint64, units of the
- * row sum) and alias [N][m] (host, nullable) of the alias table (R10). */
+ * row sum) and alias [N][m] (host, nullable) of the alias table (R10).
+ * Centralized filter: one row of m (sum <= m 2^22), device-wide passes. */
 pf_status pf_debug_resample(pf_handle* h, const uint32_t* q, const uint32_t* ua, const uint32_t* ub,
                             int32_t* ancestors, uint64_t* prob, int32_t* alias);
 

@@ -81,6 +81,147 @@ __global__ void __launch_bounds__(1024) cz_tile_prefix(const u64* __restrict__ t
     }
 }
 
+// ---- Vose over all M slots (§VI-F; the sweep closed form of
+// reading R10, device-wide): a_j = M q_j, small L = {a_j < Q} and large H
+// (both ascending), D = inclusive deficits (Q - a) over L, E = inclusive
+// excesses (a - Q) over H.  Three passes over the tiles + one prefix:
+//   vz_class   per tile: small flags, inclusive small counts / deficits
+//   (prefix)   tile totals -> inclusive prefixes
+//   vz_lists   global list positions: L[ls] = j with D, H[j - ls] = j with E
+//   vz_table   per slot: prob / alias by binary search in the other list
+// q_j is recovered from the per-tile inclusive sums cl of cz_tile_scan.
+
+__device__ __forceinline__ u64 q_of(const u64* __restrict__ cl, long long j) {
+  return (j % kCentralTile) == 0 ? cl[j] : cl[j] - cl[j - 1];
+}
+
+// block inclusive scan of a (count, sum) pair: returns the exclusive offsets
+__device__ __forceinline__ void block_excl_scan2(u64 c, u64 d, u64* sm, u64& oc, u64& od, u64& tc, u64& td) {
+  oc = block_excl_scan(c, sm, tc);
+  od = block_excl_scan(d, sm, td);
+}
+
+__global__ void __launch_bounds__(kScanThreads) vz_class(const CentralParams C) {
+  __shared__ u64 sm[32];
+  const long long M = C.M;
+  const u64 Q = C.tile_incl[M / kCentralTile - 1];
+  const long long base = static_cast<long long>(blockIdx.x) * kCentralTile + threadIdx.x * kPerThread;
+  uint32_t rc[kPerThread];
+  u64 rd[kPerThread];
+  uint32_t cnt = 0;
+  u64 dsum = 0;
+#pragma unroll
+  for (int j = 0; j < kPerThread; ++j) {
+    const u64 a = static_cast<u64>(M) * q_of(C.cl, base + j);
+    if (a < Q) {
+      ++cnt;
+      dsum += Q - a;
+    }
+    rc[j] = cnt;
+    rd[j] = dsum;
+  }
+  u64 oc, od, tc, td;
+  block_excl_scan2(cnt, dsum, sm, oc, od, tc, td);
+#pragma unroll
+  for (int j = 0; j < kPerThread; ++j) {
+    C.cn[base + j] = static_cast<uint32_t>(oc) + rc[j];
+    C.dl[base + j] = od + rd[j];
+  }
+  if (threadIdx.x == 0) {
+    C.tile_cnt[blockIdx.x] = tc;
+    C.tile_D[blockIdx.x] = td;
+  }
+}
+
+struct VoseSlot {
+  u64 a, def, Dinc, Einc;
+  long long ls;   // small slots before j
+  bool small;
+};
+__device__ __forceinline__ VoseSlot vose_slot(const CentralParams& C, long long j, u64 Q) {
+  const long long M = C.M;
+  const long long t = j / kCentralTile;
+  VoseSlot v;
+  const u64 q = q_of(C.cl, j);
+  v.a = static_cast<u64>(M) * q;
+  v.small = v.a < Q;
+  v.def = v.small ? Q - v.a : 0ull;
+  const u64 cnt_incl = (t > 0 ? C.tile_cnt_incl[t - 1] : 0ull) + C.cn[j];
+  v.ls = static_cast<long long>(cnt_incl) - (v.small ? 1 : 0);
+  v.Dinc = (t > 0 ? C.tile_D_incl[t - 1] : 0ull) + C.dl[j];
+  const u64 Cinc = (t > 0 ? C.tile_incl[t - 1] : 0ull) + C.cl[j];
+  // sum_{j' <= j} (a_j' - Q) = E_j - D_j  (wraps harmlessly in u64)
+  v.Einc = v.Dinc + static_cast<u64>(M) * Cinc - static_cast<u64>(j + 1) * Q;
+  return v;
+}
+
+__global__ void __launch_bounds__(256) vz_lists(const CentralParams C) {
+  const long long M = C.M;
+  const u64 Q = C.tile_incl[M / kCentralTile - 1];
+  const long long nL = static_cast<long long>(C.tile_cnt_incl[M / kCentralTile - 1]);
+  for (long long j = blockIdx.x * static_cast<long long>(blockDim.x) + threadIdx.x; j < M;
+       j += static_cast<long long>(gridDim.x) * blockDim.x) {
+    const VoseSlot v = vose_slot(C, j, Q);
+    const long long pos = v.small ? v.ls : nL + (j - v.ls);
+    C.lists[pos] = static_cast<int>(j);
+    C.vals[pos] = v.small ? v.Dinc : v.Einc;
+  }
+}
+
+// first index i in [0, n) with a[i] >= x
+__device__ __forceinline__ long long first_not_less(const u64* __restrict__ a, long long n, u64 x) {
+  long long lo = 0;
+  while (n > 0) {
+    const long long half = n >> 1;
+    if (__ldg(a + lo + half) < x) {
+      lo += half + 1;
+      n -= half + 1;
+    } else {
+      n = half;
+    }
+  }
+  return lo;
+}
+// first index i in [0, n) with a[i] > x
+__device__ __forceinline__ long long first_above(const u64* __restrict__ a, long long n, u64 x) {
+  long long lo = 0;
+  while (n > 0) {
+    const long long half = n >> 1;
+    if (__ldg(a + lo + half) <= x) {
+      lo += half + 1;
+      n -= half + 1;
+    } else {
+      n = half;
+    }
+  }
+  return lo;
+}
+
+__global__ void __launch_bounds__(256) vz_table(const CentralParams C) {
+  const long long M = C.M;
+  const u64 Q = C.tile_incl[M / kCentralTile - 1];
+  const long long nL = static_cast<long long>(C.tile_cnt_incl[M / kCentralTile - 1]);
+  const u64 Dtot = C.tile_D_incl[M / kCentralTile - 1];
+  for (long long j = blockIdx.x * static_cast<long long>(blockDim.x) + threadIdx.x; j < M;
+       j += static_cast<long long>(gridDim.x) * blockDim.x) {
+    const VoseSlot v = vose_slot(C, j, Q);
+    u64 pr;
+    int al;
+    if (v.small) {
+      pr = v.a;
+      al = C.lists[nL + first_not_less(C.vals + nL, M - nL, v.Dinc - v.def)];
+    } else if (v.Einc < Dtot) {
+      pr = Q + v.Einc - C.vals[first_above(C.vals, nL, v.Einc)];
+      al = C.lists[nL + (j - v.ls) + 1];
+    } else {
+      pr = Q;
+      al = static_cast<int>(j);
+    }
+    C.prob[j] = pr;
+    C.alias[j] = al;
+  }
+}
+
 // first index i in [0, n) with a[i] > x (n if none)
 __device__ __forceinline__ long long first_greater(const u64* __restrict__ a, long long n, u64 x) {
   long long lo = 0;
@@ -94,6 +235,51 @@ __device__ __forceinline__ long long first_greater(const u64* __restrict__ a, lo
     }
   }
   return lo;
+}
+
+// a8 over all M slots: the ancestor of a slot from its uniforms (U_a, U_b).
+__device__ __forceinline__ long long central_ancestor(const CentralParams& C, u64 Q, int tiles, uint32_t ua,
+                                                      uint32_t ub) {
+  if (C.vose) {
+    // Vose draw (§VI-F, R10): column b = floor(U_a M / 2^32),
+    // c = floor(U_b Q / 2^32); a = b if c < prob[b] else alias[b]
+    const long long b = static_cast<long long>((static_cast<u64>(ua) * static_cast<u64>(C.M)) >> 32);
+    const u64 c = static_cast<u64>((static_cast<unsigned __int128>(ub) * Q) >> 32);
+    return c < __ldg(C.prob + b) ? b : __ldg(C.alias + b);
+  }
+  // RWS (§VI-F, R9): c = floor(U Q / 2^32), first j with C_j > c
+  const u64 c = static_cast<u64>((static_cast<unsigned __int128>(ua) * Q) >> 32);
+  const long long b = first_greater(C.tile_incl, tiles, c);
+  const u64 excl = b > 0 ? __ldg(C.tile_incl + b - 1) : 0ull;
+  return b * kCentralTile + first_greater(C.cl + b * kCentralTile, kCentralTile, c - excl);
+}
+
+// Test hook: per-tile inclusive sums of given integer weights q (instead of
+// cz_tile_scan's q from the log-weights), then the ancestors for given uniforms.
+__global__ void __launch_bounds__(kScanThreads) cz_tile_scan_q(const uint32_t* __restrict__ q, u64* __restrict__ cl,
+                                                               u64* __restrict__ tile_sum) {
+  __shared__ u64 sm[32];
+  const long long base = static_cast<long long>(blockIdx.x) * kCentralTile + threadIdx.x * kPerThread;
+  u64 run[kPerThread];
+  u64 acc = 0;
+#pragma unroll
+  for (int j = 0; j < kPerThread; ++j) {
+    acc += q[base + j];
+    run[j] = acc;
+  }
+  u64 total;
+  const u64 off = block_excl_scan(acc, sm, total);
+#pragma unroll
+  for (int j = 0; j < kPerThread; ++j) cl[base + j] = off + run[j];
+  if (threadIdx.x == 0) tile_sum[blockIdx.x] = total;
+}
+__global__ void __launch_bounds__(256) cz_draw_debug(const CentralParams C, const uint32_t* __restrict__ ua,
+                                                     const uint32_t* __restrict__ ub, int* __restrict__ anc) {
+  const int tiles = static_cast<int>(C.M / kCentralTile);
+  const u64 Q = C.tile_incl[tiles - 1];
+  for (long long j = blockIdx.x * static_cast<long long>(blockDim.x) + threadIdx.x; j < C.M;
+       j += static_cast<long long>(gridDim.x) * blockDim.x)
+    anc[j] = static_cast<int>(central_ancestor(C, Q, tiles, ua[j], ub[j]));
 }
 
 template <int NJ>
@@ -120,14 +306,7 @@ __global__ void __launch_bounds__(256) cz_step(const CentralParams C) {
       continue;
     }
     const u32x4 b0 = philox4x32_10_rk(p, C.k, 0u, 0u, C.rk);
-    long long a = i;
-    if (!C.first) {
-      // RWS (§VI-F, R9): c = floor(U Q / 2^32), first j with C_j > c
-      const u64 c = static_cast<u64>((static_cast<unsigned __int128>(b0.x) * Q) >> 32);
-      const long long b = first_greater(C.tile_incl, tiles, c);
-      const u64 excl = b > 0 ? __ldg(C.tile_incl + b - 1) : 0ull;
-      a = b * kCentralTile + first_greater(C.cl + b * kCentralTile, kCentralTile, c - excl);
-    }
+    const long long a = C.first ? i : central_ancestor(C, Q, tiles, b0.x, b0.y);
     const float* xa = C.in + a;
     auto x = [xa, M](int c) { return __ldg(xa + c * M); };
     NoiseGen gen{p, C.k, C.rk, u32x4{0u, 0u, b0.z, b0.w}};
@@ -174,6 +353,17 @@ __global__ void __launch_bounds__(256) cz_step(const CentralParams C) {
   }
 }
 
+// the alias table; Q = tile_incl[tiles - 1] is read on the device
+void vose_table(const CentralParams& c, cudaStream_t s) {
+  const int tiles = static_cast<int>(c.M / kCentralTile);
+  const int g2 = static_cast<int>(c.M / 256 < 148 * 8 ? c.M / 256 : 148 * 8);
+  vz_class<<<tiles, kScanThreads, 0, s>>>(c);
+  cz_tile_prefix<<<1, 1024, 0, s>>>(c.tile_cnt, c.tile_cnt_incl, tiles);
+  cz_tile_prefix<<<1, 1024, 0, s>>>(c.tile_D, c.tile_D_incl, tiles);
+  vz_lists<<<g2, 256, 0, s>>>(c);
+  vz_table<<<g2, 256, 0, s>>>(c);
+}
+
 template <int NJ>
 cudaError_t central_step_nj(const CentralParams& c, int grid, cudaStream_t s) {
   const int tiles = static_cast<int>(c.M / kCentralTile);
@@ -181,6 +371,7 @@ cudaError_t central_step_nj(const CentralParams& c, int grid, cudaStream_t s) {
     cz_tile_scan<<<tiles, kScanThreads, 0, s>>>(c.in + static_cast<long long>(NJ + 4) * c.M, c.record_prev, c.cl,
                                                 c.tile_sum);
     cz_tile_prefix<<<1, 1024, 0, s>>>(c.tile_sum, c.tile_incl, tiles);
+    if (c.vose) vose_table(c, s);
   }
   cz_step<NJ><<<grid, 256, 0, s>>>(c);
   return cudaGetLastError();
@@ -195,6 +386,16 @@ cudaError_t central_step(int nj, const CentralParams& c, int grid, cudaStream_t 
     case 28: return central_step_nj<28>(c, grid, s);
     default: return cudaErrorInvalidValue;
   }
+}
+
+cudaError_t central_resample_debug(const CentralParams& c, const uint32_t* q, const uint32_t* ua, const uint32_t* ub,
+                                   int* anc, cudaStream_t s) {
+  const int tiles = static_cast<int>(c.M / kCentralTile);
+  cz_tile_scan_q<<<tiles, kScanThreads, 0, s>>>(q, c.cl, c.tile_sum);
+  cz_tile_prefix<<<1, 1024, 0, s>>>(c.tile_sum, c.tile_incl, tiles);
+  if (c.vose) vose_table(c, s);
+  cz_draw_debug<<<static_cast<int>(c.M / 256 < 148 * 8 ? c.M / 256 : 148 * 8), 256, 0, s>>>(c, ua, ub, anc);
+  return cudaGetLastError();
 }
 
 int central_grid(int nj, int sms) {

@@ -33,9 +33,29 @@ struct CentralParams {
   uint32_t k;
   int first;     // k == 1 (or the sample-only test hook): no resampling
   int publish;   // only the argmax / record of the set in `in` (checkpoint restore)
+  // Vose (resampler 1): the alias table over all M slots (sweep closed form, R10)
+  int vose;
+  unsigned long long* dl;          // [M] per-tile inclusive deficit sums over the small slots
+  uint32_t* cn;                    // [M] per-tile inclusive small-slot counts
+  int* lists;                      // [M] small slots ascending, then large slots ascending
+  unsigned long long* vals;        // [M] D over the small list, then E over the large list
+  unsigned long long* prob;        // [M] alias-table threshold (units of Q / M)
+  int* alias;                      // [M]
+  unsigned long long* tile_cnt;    // [tiles] small count per tile, then its inclusive prefix
+  unsigned long long* tile_cnt_incl;
+  unsigned long long* tile_D;      // [tiles] deficit sum per tile, then its inclusive prefix
+  unsigned long long* tile_D_incl;
 };
 
+// Largest centralized filter resampled by Vose: the deficit / excess sums
+// (<= M Q <= M^2 2^22) stay below 2^64.
+constexpr long long kCentralVoseMax = 1ll << 20;
+
 cudaError_t central_step(int nj, const CentralParams& c, int grid, cudaStream_t s);
+// test hook: RWS / Vose ancestors over all M slots from integer weights q [M]
+// and uniforms ua, ub [M] (device); the Vose table is left in c.prob / c.alias
+cudaError_t central_resample_debug(const CentralParams& c, const uint32_t* q, const uint32_t* ua, const uint32_t* ub,
+                                   int* anc, cudaStream_t s);
 int central_grid(int nj, int sms);
 
 }  // namespace pf

@@ -90,6 +90,7 @@ struct Geometry {
   int nj, d, m, deg, tt, E;
   long long N, R, C, n_local, g0, n_ext, M_local, ROW;
   bool central;   // one filter of m > 1024 particles, resampled globally (pf_central.cu)
+  bool vose;      // resampler (central filter sizing)
   long long tiles;
 };
 
@@ -104,10 +105,13 @@ pf_status validate(const pf_config* cfg, const pf_model_params* mp, Geometry* g)
     return PF_EINVAL;
   // Centralized filter (NEXT-2): a single filter of M > 1024 particles.
   g->central = cfg->n_filters == 1 && m > 1024;
+  g->vose = false;
   if (g->central) {
     if (m % pf::kCentralTile != 0 || m > (1 << 26) || cfg->world != 1) return PF_EINVAL;
     if (cfg->topo != PF_TOPO_NONE && cfg->t != 0) return PF_EINVAL;
-    if (cfg->resampler != PF_RESAMPLE_RWS) return PF_EUNSUPPORTED;
+    if (cfg->resampler != PF_RESAMPLE_RWS && cfg->resampler != PF_RESAMPLE_VOSE) return PF_EINVAL;
+    if (cfg->resampler == PF_RESAMPLE_VOSE && m > pf::kCentralVoseMax) return PF_EUNSUPPORTED;
+    g->vose = cfg->resampler == PF_RESAMPLE_VOSE;
     if (mp->n_joints != 2 && mp->n_joints != 5 && mp->n_joints != 28) return PF_EUNSUPPORTED;
     g->nj = mp->n_joints;
     g->d = mp->n_joints + 4;
@@ -268,8 +272,11 @@ void host_inputs(pf_handle* h, pf::StepParams& p, const float* z, const float* u
 
 // Centralized filter: particle buffers ping-pong ([2][D+1][M]), then the
 // per-particle tile sums (u64 [M]) and two u64 arrays of tile totals.
+// Vose adds per slot dl, vals, prob (u64) and cn, lists, alias (32-bit), and
+// four u64 arrays of tile totals / prefixes.
 size_t central_bytes(const Geometry& g) {
-  return sizeof(float) * 2 * g.ROW + sizeof(u64) * (g.M_local + 2 * g.tiles);
+  const size_t vose = g.vose ? sizeof(u64) * (3 * g.M_local + 4 * g.tiles) + sizeof(uint32_t) * 3 * g.M_local : 0;
+  return sizeof(float) * 2 * g.ROW + sizeof(u64) * (g.M_local + 2 * g.tiles) + vose;
 }
 // weighted set of step k lives in particle buffer (central: k & 1; else the only one)
 float* set_of_step(pf_handle* h, long long k) { return h->parts + (h->g.central ? (k & 1) * h->g.ROW : 0); }
@@ -285,6 +292,22 @@ pf::CentralParams central_params(pf_handle* h, long long k) {
   c.cl = aux;
   c.tile_sum = aux + h->g.M_local;
   c.tile_incl = aux + h->g.M_local + h->g.tiles;
+  if (h->g.vose) {
+    const long long M = h->g.M_local, T = h->g.tiles;
+    u64* v = aux + M + 2 * T;
+    c.vose = 1;
+    c.dl = v;
+    c.vals = v + M;
+    c.prob = v + 2 * M;
+    c.tile_cnt = v + 3 * M;
+    c.tile_cnt_incl = v + 3 * M + T;
+    c.tile_D = v + 3 * M + 2 * T;
+    c.tile_D_incl = v + 3 * M + 3 * T;
+    uint32_t* w = reinterpret_cast<uint32_t*>(v + 3 * M + 4 * T);
+    c.cn = w;
+    c.lists = reinterpret_cast<int*>(w + M);
+    c.alias = reinterpret_cast<int*>(w + 2 * M);
+  }
   c.key_cur = keys(h) + (k & 1);
   c.key_next = keys(h) + ((k + 1) & 1);
   c.counter = reinterpret_cast<unsigned int*>(h->scratch + kOffCounter);
@@ -715,7 +738,6 @@ pf_status pf_debug_resample(pf_handle* h, const uint32_t* q, const uint32_t* ua,
                             int32_t* ancestors, uint64_t* prob, int32_t* alias) {
   if (!h || !q || !ua || !ub || !ancestors) return PF_EINVAL;
   if (h->err != PF_OK) return h->err;
-  if (h->g.central) return PF_ESTATE;
   const long long n = h->g.N * h->g.m;
   DevBuf<uint32_t> dq, dua, dub;
   DevBuf<int> danc, dal;
@@ -731,9 +753,16 @@ pf_status pf_debug_resample(pf_handle* h, const uint32_t* q, const uint32_t* ua,
   if (e == cudaSuccess) e = cudaMemcpy(dq.p, q, 4 * n, cudaMemcpyHostToDevice);
   if (e == cudaSuccess) e = cudaMemcpy(dua.p, ua, 4 * n, cudaMemcpyHostToDevice);
   if (e == cudaSuccess) e = cudaMemcpy(dub.p, ub, 4 * n, cudaMemcpyHostToDevice);
-  if (e == cudaSuccess)
+  if (e == cudaSuccess && h->g.central) {
+    // one filter over all M slots (clobbers the handle's scan / table arrays)
+    const pf::CentralParams c = central_params(h, h->step + 1);
+    e = pf::central_resample_debug(c, dq.p, dua.p, dub.p, danc.p, h->stream);
+    if (e == cudaSuccess && want_table) e = cudaMemcpyAsync(dpr.p, c.prob, 8 * n, cudaMemcpyDeviceToDevice, h->stream);
+    if (e == cudaSuccess && want_table) e = cudaMemcpyAsync(dal.p, c.alias, 4 * n, cudaMemcpyDeviceToDevice, h->stream);
+  } else if (e == cudaSuccess) {
     e = h->ke->resample_debug(dq.p, dua.p, dub.p, danc.p, want_table ? dpr.p : nullptr, want_table ? dal.p : nullptr,
                               h->g.N, h->stream);
+  }
   if (e == cudaSuccess) e = cudaStreamSynchronize(h->stream);
   if (e == cudaSuccess) e = cudaMemcpy(ancestors, danc.p, 4 * n, cudaMemcpyDeviceToHost);
   if (e == cudaSuccess && want_table) e = cudaMemcpy(prob, dpr.p, 8 * n, cudaMemcpyDeviceToHost);

@@ -19,19 +19,20 @@ def P():
     return F
 
 
-def _pair(P, orc, W, nj, M, seed, T=12, traj_seed=0):
+def _pair(P, orc, W, nj, M, seed, T=12, traj_seed=0, res="rws"):
     tr = W.make_trajectory(nj, T, traj_seed)
     g = P.ParticleFilter(tr["mu0"], tr["sigma0"], P.ArmModel(n_joints=nj), m=M, n_filters=1, t=0, topo="none",
-                         resampler="rws", seed=seed)
-    o = orc.Filter(orc.Config(m=M, n_filters=1, t=0, topo="none", resampler="rws", seed=seed),
+                         resampler=res, seed=seed)
+    o = orc.Filter(orc.Config(m=M, n_filters=1, t=0, topo="none", resampler=res, seed=seed),
                    orc.Model(n_joints=nj), tr["mu0"], tr["sigma0"])
     return tr, g, o
 
 
-@pytest.mark.parametrize("nj,M", [(2, 4096), (5, 8192), (28, 4096), (5, 12288)])
-def test_central_trajectory_bit_exact(P, orc, W, nj, M):
+@pytest.mark.parametrize("nj,M,res", [(2, 4096, "rws"), (5, 8192, "rws"), (28, 4096, "rws"), (5, 12288, "rws"),
+                                      (5, 8192, "vose"), (2, 12288, "vose"), (28, 4096, "vose")])
+def test_central_trajectory_bit_exact(P, orc, W, nj, M, res):
     # several scan tiles (4096) and, for 12288, a non-power-of-two tile count
-    tr, g, o = _pair(P, orc, W, nj, M, seed=nj * 7 + M)
+    tr, g, o = _pair(P, orc, W, nj, M, seed=nj * 7 + M, res=res)
     for k in range(1, 9):
         g.step(tr["Z"][k], tr["U"][k - 1])
         o.step(tr["Z"][k], tr["U"][k - 1])
@@ -87,14 +88,15 @@ def test_central_resume_and_batch(P, orc, W):
     g.close()
 
 
-@pytest.mark.parametrize("nj,M", [(5, 1 << 20), (5, 1 << 22), (28, 1 << 20)])
-def test_central_full_size_sampled(P, orc, W, nj, M):
+@pytest.mark.parametrize("nj,M,res", [(5, 1 << 20, "rws"), (5, 1 << 22, "rws"), (28, 1 << 20, "rws"),
+                                      (5, 1 << 20, "vose")])
+def test_central_full_size_sampled(P, orc, W, nj, M, res):
     # full size (the paper's centralized curves reach 2^20 particles, Fig. 5):
     # one step from a generator-made weighted set; the oracle recomputes a
     # sample of slots one by one (normalise over all M, RWS, sample, weight)
     tr = W.make_trajectory(nj, 10, 2)
     g = P.ParticleFilter(tr["mu0"], tr["sigma0"], P.ArmModel(n_joints=nj), m=M, n_filters=1, t=0, topo="none",
-                         seed=4242)
+                         seed=4242, resampler=res)
     s0 = W.random_particles(tr, M, 5)
     w0 = W.random_logw(1, M, 5).ravel()
     g.set_particles(s0, w0, 4)
@@ -103,7 +105,7 @@ def test_central_full_size_sampled(P, orc, W, nj, M):
     assert k == 5
     rng = np.random.default_rng(M + nj)
     slots = np.unique(np.concatenate([[0, 1, 4095, 4096, M // 2, M - 1], rng.integers(0, M, 58)]))
-    cfg = orc.Config(m=M, n_filters=1, t=0, topo="none", resampler="rws", seed=4242)
+    cfg = orc.Config(m=M, n_filters=1, t=0, topo="none", resampler=res, seed=4242)
     so, wo = orc.central_slots(cfg, orc.Model(n_joints=nj), s0, w0, 5, tr["Z"][5], tr["U"][4], slots)
     np.testing.assert_array_equal(sg[:, slots], so)
     np.testing.assert_array_equal(wg[slots], wo)
@@ -121,10 +123,53 @@ def test_central_errors(P, W):
     with pytest.raises(B.PFError):
         mk(m=5000)                       # not a multiple of the 4096-particle scan tile
     with pytest.raises(B.PFError):
-        mk(m=8192, resampler="vose")     # centralized Vose: not built
+        mk(m=1 << 21, resampler="vose")  # centralized Vose: u64 alias sums need m <= 2^20
     g = mk(m=4096)
-    q = np.zeros(4096, np.uint32)
-    assert B.lib().pf_debug_resample(g.h, q.ctypes.data, q.ctypes.data, q.ctypes.data, q.ctypes.data, None,
-                                     None) == B.PF_ESTATE
     assert B.lib().pf_set_trace(g.h, 1) == B.PF_ESTATE
     g.close()
+
+
+@pytest.mark.parametrize("M", [8192, 12288])
+@pytest.mark.parametrize("kind", ["mixed", "uniform", "onehot", "sparse"])
+def test_central_resample_tables_bit_exact(P, orc, W, M, kind):
+    # the device-wide RWS search and Vose table (closed form over all M slots,
+    # R10) against the oracle's sequential sum / sequential sweep, slot by slot
+    from paper_conf_ipps_chitchianasks13_b200 import binding as B
+    rng = np.random.default_rng(M + len(kind))
+    if kind == "mixed":
+        q = rng.integers(0, 1 << 22, M).astype(np.uint32)
+        q[rng.random(M) < 0.3] = 0
+    elif kind == "uniform":
+        q = np.full(M, 1 << 22, np.uint32)
+    elif kind == "onehot":
+        q = np.zeros(M, np.uint32)
+        q[M // 3] = 1 << 22
+    else:
+        q = np.zeros(M, np.uint32)
+        q[rng.integers(0, M, 17)] = rng.integers(1, 1 << 22, 17).astype(np.uint32)
+    ua = rng.integers(0, 2**32, M, dtype=np.uint64).astype(np.uint32)
+    ub = rng.integers(0, 2**32, M, dtype=np.uint64).astype(np.uint32)
+    ua[:3] = [0, 0xFFFFFFFF, 0x80000000]
+    ub[:3] = [0, 0xFFFFFFFF, 0x7FFFFFFF]
+    tr = W.make_trajectory(5, 3, 0)
+    for res in ("rws", "vose"):
+        g = P.ParticleFilter(tr["mu0"], tr["sigma0"], P.ArmModel(n_joints=5), m=M, n_filters=1, t=0, topo="none",
+                             resampler=res)
+        anc = np.zeros(M, np.int32)
+        prob = np.zeros(M, np.uint64)
+        alias = np.zeros(M, np.int32)
+        B.pf_debug_resample(g.h, q, ua, ub, anc, prob if res == "vose" else None, alias if res == "vose" else None)
+        g.close()
+        if res == "vose":
+            pr, al = orc.vose_build(q)
+            np.testing.assert_array_equal(prob, pr)
+            np.testing.assert_array_equal(alias, al)
+            Q = int(q.astype(np.uint64).sum())
+            mass = prob.copy()   # alias mass of slot j = prob_j + sum over columns aliasing j of (Q - prob)
+            np.add.at(mass, alias, np.uint64(Q) - prob)
+            np.testing.assert_array_equal(mass, np.uint64(M) * q.astype(np.uint64))
+            ref = np.array([orc.vose_draw(pr, al, Q, int(a), int(b)) for a, b in zip(ua, ub)], np.int32)
+        else:
+            ref = np.array([orc.rws_draw(q, int(a)) for a in ua], np.int32)
+        np.testing.assert_array_equal(anc, ref)
+        assert np.all(q[anc] > 0)   # never a zero-weight slot
