@@ -62,6 +62,20 @@ typedef enum { PF_MODEL_ARM_PLANAR = 0 } pf_model_id;
 /* pf_config.flags */
 #define PF_DEVICE_INPUTS 1u   /* pf_step's z / u are device pointers         */
 
+/* When a sub-filter resamples (§IV: "we have experimented with
+ * the suggested metric to compute the effective sample size as well as a
+ * simpler resampling frequency parameter (each sub-filter randomly decides to
+ * resample at a fixed ratio of the time)"; reading R21).  A sub-filter that
+ * does not resample keeps its particles and carries its normalised
+ * log-weight l - l_max into the next weight (F12). */
+typedef enum {
+  PF_POLICY_ALWAYS = 0,   /* resample every step (the paper's choice)                     */
+  PF_POLICY_ESS = 1,      /* resample iff Q^2 2^16 < param m sum q^2 (ESS < tau m, tau =   */
+                          /* param / 2^16; q = the integer weights of F7, exact integers)  */
+  PF_POLICY_FREQ = 2      /* resample iff word 0 of Philox (n, k, 1, 0) < param            */
+                          /* (param = ratio 2^32 in [0, 2^32])                             */
+} pf_policy;
+
 typedef struct {
   int32_t model;            /* pf_model_id                                           */
   int32_t n_joints;         /* joints incl. base rotation; d = n_joints + 4          */
@@ -92,6 +106,8 @@ typedef struct {
   int32_t rank;             /* shard index in [0, world)                             */
   int32_t world;            /* number of shards (processes / GPUs), >= 1             */
   uint32_t flags;           /* PF_DEVICE_INPUTS                                      */
+  int32_t resample_policy;  /* pf_policy (sub-filters; the centralized filter: ALWAYS) */
+  uint64_t resample_param;  /* see pf_policy; <= 2^32                                */
 } pf_config;
 
 /* Bytes of each caller-owned device buffer. */

@@ -41,6 +41,11 @@ extern "C" {
 
 enum { ORC_TOPO_NONE = 0, ORC_TOPO_RING = 1, ORC_TOPO_TORUS2D = 2, ORC_TOPO_ALL2ALL = 3 };
 enum { ORC_RWS = 0, ORC_VOSE = 1 };
+/* When a sub-filter resamples (§IV: "the suggested metric to
+ * compute the effective sample size as well as a simpler resampling frequency
+ * parameter (each sub-filter randomly decides to resample at a fixed ratio of
+ * the time)"; reading R21). */
+enum { ORC_POLICY_ALWAYS = 0, ORC_POLICY_ESS = 1, ORC_POLICY_FREQ = 2 };
 
 /* Table I parameters: m, N, X, t; plus the RNG seed. */
 typedef struct {
@@ -52,7 +57,16 @@ typedef struct {
   int32_t torus_cols;   /* 0 = default N / R                               */
   int32_t resampler;    /* ORC_RWS | ORC_VOSE                              */
   uint64_t seed;        /* Philox key = (seed lo 32, seed hi 32)  (R12)    */
+  int32_t policy;       /* ORC_POLICY_*                                    */
+  uint64_t policy_param;/* ESS: tau in 1/65536 of m; FREQ: threshold in [0, 2^32] */
 } orc_config;
+
+/* R21: does sub-filter n (global) resample before the sample of step k?
+ * q = its integer weights (F7).  ESS: Q^2 2^16 < param m S2 (Q = sum q,
+ * S2 = sum q^2, i.e. ESS = Q^2/S2 < tau m; 128-bit integers); FREQ: word 0 of
+ * Philox (n, k, 1, 0) < param. */
+int orc_should_resample(int32_t policy, uint64_t param, const uint32_t* q, int32_t m, uint64_t seed, int64_t n,
+                        int64_t k);
 
 /* Table II model parameters (§VII-A) — fp32 values. */
 typedef struct {

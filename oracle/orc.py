@@ -20,6 +20,17 @@ SOURCES = [os.path.join(HERE, f) for f in ("orc.c", "orc_impl.inc", "orc.h")]
 
 TOPO = {"none": 0, "ring": 1, "torus": 2, "all2all": 3}
 RESAMPLER = {"rws": 0, "vose": 1}
+POLICY = {"always": 0, "ess": 1, "freq": 2}
+
+
+def policy_param(policy: str, value: float) -> int:
+    """R21 integer parameter: ESS threshold tau (fraction of m) in 1/65536;
+    resampling ratio in [0, 1] as a threshold on a 32-bit Philox word."""
+    if policy == "ess":
+        return int(round(value * 65536))
+    if policy == "freq":
+        return min(1 << 32, max(0, int(round(value * 2.0**32))))
+    return 0
 
 CFLAGS = ["-O2", "-std=c11", "-Wall", "-ffp-contract=off", "-fno-fast-math", "-fPIC", "-shared"]
 
@@ -38,7 +49,7 @@ def build(force: bool = False) -> str:
 class OrcConfig(C.Structure):
     _fields_ = [("m", C.c_int32), ("n_filters", C.c_int64), ("t", C.c_int32), ("topo", C.c_int32),
                 ("torus_rows", C.c_int32), ("torus_cols", C.c_int32), ("resampler", C.c_int32),
-                ("seed", C.c_uint64)]
+                ("seed", C.c_uint64), ("policy", C.c_int32), ("policy_param", C.c_uint64)]
 
 
 class OrcModel(C.Structure):
@@ -73,6 +84,8 @@ def lib():
             "orc_d_sample_weight": (None, [P, C.c_uint64, C.c_int64, C.c_int64, P, P, P, C.c_int64, P, P]),
             "orc_rws_draw": (C.c_int32, [P, C.c_int32, C.c_uint32]),
             "orc_vose_build": (None, [P, C.c_int32, P, P]),
+            "orc_should_resample": (C.c_int, [C.c_int32, C.c_uint64, P, C.c_int32, C.c_uint64, C.c_int64,
+                                              C.c_int64]),
             "orc_vose_draw": (C.c_int32, [P, P, C.c_int32, C.c_uint64, C.c_uint32, C.c_uint32]),
             "orc_resample_q": (C.c_int, [P, C.c_int64, C.c_int32, C.c_int32, P, P, P]),
             "orc_s_normalise": (None, [P, C.c_int32, P]),
@@ -151,10 +164,13 @@ class Config:
     seed: int = 0
     torus_rows: int = 0
     torus_cols: int = 0
+    policy: str = "always"     # R21: "always" | "ess" | "freq"
+    policy_param: int = 0      # ess: tau * 2^16; freq: ratio * 2^32 (integers, see policy_param())
 
     def c(self) -> OrcConfig:
         return OrcConfig(self.m, self.n_filters, self.t, TOPO[self.topo], self.torus_rows,
-                         self.torus_cols, RESAMPLER[self.resampler], self.seed)
+                         self.torus_cols, RESAMPLER[self.resampler], self.seed, POLICY[self.policy],
+                         self.policy_param)
 
 
 # ---- component functions --------------------------------------------------
@@ -233,6 +249,11 @@ def sample_weight(model: Model, seed: int, state_in, z, u, k: int, p_offset: int
 def rws_draw(q, U: int) -> int:
     qq = _u32(q)
     return lib().orc_rws_draw(_p(qq), len(qq), U)
+
+
+def should_resample(policy: str, param: int, q, seed: int, n: int, k: int) -> bool:
+    qq = _u32(q)
+    return bool(lib().orc_should_resample(POLICY[policy], param, _p(qq), len(qq), seed, n, k))
 
 
 def vose_build(q):

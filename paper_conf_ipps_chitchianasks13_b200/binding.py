@@ -16,6 +16,7 @@ LIB_PATH = os.environ.get("PF_LIB") or os.path.join(HERE, "libpf_b200.so")   # P
 PF_OK, PF_EINVAL, PF_ENOMEM, PF_ECUDA, PF_ESTATE, PF_EUNSUPPORTED = 0, -1, -2, -3, -5, -6
 PF_TOPO_NONE, PF_TOPO_RING, PF_TOPO_TORUS2D, PF_TOPO_ALL2ALL = 0, 1, 2, 3
 PF_RESAMPLE_RWS, PF_RESAMPLE_VOSE = 0, 1
+PF_POLICY_ALWAYS, PF_POLICY_ESS, PF_POLICY_FREQ = 0, 1, 2
 PF_MODEL_ARM_PLANAR = 0
 PF_DEVICE_INPUTS = 1
 
@@ -37,7 +38,8 @@ class pf_model_params(C.Structure):
 class pf_config(C.Structure):
     _fields_ = [("m", C.c_int32), ("n_filters", C.c_int64), ("t", C.c_int32), ("topo", C.c_int32),
                 ("torus_rows", C.c_int32), ("torus_cols", C.c_int32), ("resampler", C.c_int32),
-                ("seed", C.c_uint64), ("rank", C.c_int32), ("world", C.c_int32), ("flags", C.c_uint32)]
+                ("seed", C.c_uint64), ("rank", C.c_int32), ("world", C.c_int32), ("flags", C.c_uint32),
+                ("resample_policy", C.c_int32), ("resample_param", C.c_uint64)]
 
 
 class pf_sizes(C.Structure):

@@ -41,6 +41,7 @@ typedef unsigned long long u64;
 enum : int { MODE_STEP = 0, MODE_PUBLISH = 1, MODE_EXCHANGE = 2, MODE_SAMPLE = 3 };
 enum : int { TOPO_NONE = 0, TOPO_RING = 1, TOPO_TORUS = 2, TOPO_A2A = 3 };
 enum : int { RES_RWS = 0, RES_VOSE = 1 };
+enum : int { POLICY_ALWAYS = 0, POLICY_ESS = 1, POLICY_FREQ = 2 };
 
 struct StepParams {
   ArmConsts mc;
@@ -66,6 +67,8 @@ struct StepParams {
   uint32_t t_inv;          // ceil(2^16 / t): lane / t = (lane * t_inv) >> 16 for lane < 2^16 / t
   uint32_t k;
   int mode, first;
+  int policy;              // R21: POLICY_ALWAYS / _ESS / _FREQ
+  unsigned long long policy_param;   // ESS: tau 2^16; FREQ: threshold on a Philox word
   uint32_t rk[20];         // Philox round keys (key0 + r W0, key1 + r W1), r = 0..9
   float zin[32];           // step inputs carried by the launch itself (host-input mode)
   float uin[32];
@@ -201,6 +204,24 @@ __device__ __forceinline__ u64 gmax_u64(u64 v, GroupCtx& G) {
     if (G.lane == 0) r[G.wig] = w;
     gsync<GW>(G.g);
     return warp_max_u64(G.lane < GW ? r[G.lane] : 0ull);
+  }
+}
+
+template <int GW>
+__device__ __forceinline__ u64 gsum_u64(u64 v, GroupCtx& G) {
+#pragma unroll
+  for (int o = 16; o >= 1; o >>= 1) v += __shfl_xor_sync(0xFFFFFFFFu, v, o);
+  if constexpr (GW == 1) {
+    return v;
+  } else {
+    u64* r = G.red + G.rb * 32;
+    G.rb ^= 1;
+    if (G.lane == 0) r[G.wig] = v;
+    gsync<GW>(G.g);
+    u64 t = 0;
+#pragma unroll
+    for (int w = 0; w < GW; ++w) t += r[w];
+    return t;
   }
 }
 
@@ -778,6 +799,8 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
     // ---- a7 normalise + a8 resample (slot order, R11)
     int anc[PP];
     uint32_t bz[PP], bw[PP];   // Philox block 0, words 2-3 (first Box–Muller pair)
+    bool resampled = true;     // false: conditional policy kept the set (R21)
+    float carry[PP];
     {
       uint32_t ua[PP], ub[PP], q[PP];
 #pragma unroll
@@ -811,7 +834,27 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
         const float lmax = unord_f32(lmax_o);
 #pragma unroll
         for (int j = 0; j < PP; ++j) q[j] = expq_c(lw[j] - lmax);
-        resample_group<C>(q, ua, ub, anc, S, G, nullptr, nullptr);
+        // R21: does this sub-filter resample now?  (uniform in the group)
+        if (P.policy == POLICY_ESS) {   // ESS = Q^2 / sum q^2 < tau m, exactly in integers
+          u64 s1 = 0, s2 = 0;
+#pragma unroll
+          for (int j = 0; j < PP; ++j) {
+            s1 += q[j];
+            s2 += static_cast<u64>(q[j]) * q[j];
+          }
+          const u64 Qs = gsum_u64<GW>(s1, G), S2 = gsum_u64<GW>(s2, G);
+          resampled = ((static_cast<unsigned __int128>(Qs) * Qs) << 16) <
+                      static_cast<unsigned __int128>(P.policy_param) * static_cast<u64>(M) * S2;
+        } else if (P.policy == POLICY_FREQ) {   // a coin per (sub-filter, step): Philox stream 1
+          resampled = static_cast<u64>(philox4x32_10_rk(static_cast<uint32_t>(gsf), P.k, 1u, 0u, P.rk).x) <
+                      P.policy_param;
+        }
+        if (resampled) {
+          resample_group<C>(q, ua, ub, anc, S, G, nullptr, nullptr);
+        } else {   // keep the particles, carry l - l_max into the next weight (F12)
+#pragma unroll
+          for (int j = 0; j < PP; ++j) carry[j] = lw[j] - lmax;
+        }
       }
       if (mode == MODE_STEP && P.dbg_anc) {
 #pragma unroll
@@ -825,7 +868,11 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
 #pragma unroll
         for (int j = 0; j < PP; ++j) {
           const int s = C::slot(G.t, j);
-          reinterpret_cast<int*>(ws)[s] = anc[j];
+          if (resampled) {
+            reinterpret_cast<int*>(ws)[s] = anc[j];
+          } else {
+            ws[s] = carry[j];   // ancestor = own slot
+          }
           bzw_s[s] = make_uint2(bz[j], bw[j]);
         }
       }
@@ -840,9 +887,17 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
         const int sa = C::slot(G.t, j), sb = C::slot(G.t, j + 1);
         int a0, a1;
         uint32_t za2, za3, zb2, zb3;
+        float c0 = 0.0f, c1 = 0.0f;
         if constexpr (C::STAGED) {
-          a0 = reinterpret_cast<const int*>(ws)[sa];
-          a1 = reinterpret_cast<const int*>(ws)[sb];
+          if (resampled) {
+            a0 = reinterpret_cast<const int*>(ws)[sa];
+            a1 = reinterpret_cast<const int*>(ws)[sb];
+          } else {
+            a0 = sa;
+            a1 = sb;
+            c0 = ws[sa];
+            c1 = ws[sb];
+          }
           const uint2 pa = bzw_s[sa], pb = bzw_s[sb];
           za2 = pa.x;
           za3 = pa.y;
@@ -851,6 +906,10 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
         } else {
           a0 = anc[j];
           a1 = anc[j + 1];
+          if (!resampled) {
+            c0 = carry[j];
+            c1 = carry[j + 1];
+          }
           za2 = bz[j];
           za3 = bw[j];
           zb2 = bz[j + 1];
@@ -868,7 +927,8 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
           outa[c * M] = lo2(v);
           outb[c * M] = hi2(v);
         });
-        const f2 l = arm_finish2(P.mc2, z2_s, A);
+        f2 l = arm_finish2(P.mc2, z2_s, A);
+        if (!resampled) l = add2(pk(c0, c1), l);   // F12
         outa[D * M] = lo2(l);
         outb[D * M] = hi2(l);
         reinterpret_cast<float*>(bzw_s)[2 * sa] = lo2(l);   // own slots, after their Philox words were read
@@ -883,13 +943,20 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
         const int s = C::slot(G.t, j);
         int a;
         uint32_t z2, z3;
+        float cr = 0.0f;
         if constexpr (C::STAGED) {
-          a = reinterpret_cast<const int*>(ws)[s];
+          if (resampled) {
+            a = reinterpret_cast<const int*>(ws)[s];
+          } else {
+            a = s;
+            cr = ws[s];
+          }
           const uint2 bb = bzw_s[s];
           z2 = bb.x;
           z3 = bb.y;
         } else {
           a = anc[j];
+          if (!resampled) cr = carry[j];
           z2 = bz[j];
           z3 = bw[j];
         }
@@ -899,7 +966,8 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
         NoiseGen gen{pbase + static_cast<uint32_t>(s), P.k, P.rk, u32x4{0u, 0u, z2, z3}};
         ArmAcc A;
         SampleStream<NJ, 0>::run(P.mc, hsu_s, z_s, x, gen, A, [out](int c, float v) { out[c * M] = v; });
-        const float l = arm_finish(P.mc, z_s, A);
+        float l = arm_finish(P.mc, z_s, A);
+        if (!resampled) l = cr + l;   // F12
         out[D * M] = l;
         reinterpret_cast<float*>(bzw_s)[2 * s] = l;   // own slot, after its Philox words were read
 

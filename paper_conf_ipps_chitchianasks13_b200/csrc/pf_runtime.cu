@@ -103,6 +103,9 @@ pf_status validate(const pf_config* cfg, const pf_model_params* mp, Geometry* g)
   const int m = cfg->m;
   if (cfg->n_filters < 1 || cfg->t < 0 || cfg->world < 1 || cfg->rank < 0 || cfg->rank >= cfg->world)
     return PF_EINVAL;
+  if (cfg->resample_policy < PF_POLICY_ALWAYS || cfg->resample_policy > PF_POLICY_FREQ ||
+      cfg->resample_param > (1ull << 32))
+    return PF_EINVAL;
   // Centralized filter (NEXT-2): a single filter of M > 1024 particles.
   g->central = cfg->n_filters == 1 && m > 1024;
   g->vose = false;
@@ -111,6 +114,7 @@ pf_status validate(const pf_config* cfg, const pf_model_params* mp, Geometry* g)
     if (cfg->topo != PF_TOPO_NONE && cfg->t != 0) return PF_EINVAL;
     if (cfg->resampler != PF_RESAMPLE_RWS && cfg->resampler != PF_RESAMPLE_VOSE) return PF_EINVAL;
     if (cfg->resampler == PF_RESAMPLE_VOSE && m > pf::kCentralVoseMax) return PF_EUNSUPPORTED;
+    if (cfg->resample_policy != PF_POLICY_ALWAYS) return PF_EUNSUPPORTED;
     g->vose = cfg->resampler == PF_RESAMPLE_VOSE;
     if (mp->n_joints != 2 && mp->n_joints != 5 && mp->n_joints != 28) return PF_EUNSUPPORTED;
     g->nj = mp->n_joints;
@@ -256,6 +260,8 @@ pf::StepParams base_params(pf_handle* h, long long k, int mode) {
     p.rk[2 * r + 1] = key1 + static_cast<uint32_t>(r) * 0xBB67AE85u;
   }
   p.k = static_cast<uint32_t>(k);
+  p.policy = h->cfg.resample_policy;
+  p.policy_param = h->cfg.resample_param;
   p.mode = mode;
   p.first = (k == 1) ? 1 : 0;
   return p;

@@ -38,6 +38,19 @@ class ArmModel:
                                  self.sigma_pos, self.sigma_vel, self.sigma_cam, self.sigma_theta_meas)
 
 
+POLICY = {"always": B.PF_POLICY_ALWAYS, "ess": B.PF_POLICY_ESS, "freq": B.PF_POLICY_FREQ}
+
+
+def _policy_param(policy: str, value: float) -> int:
+    """pf_config.resample_param (pf.h pf_policy): ESS tau in 1/65536 of m;
+    resampling ratio as a threshold on a 32-bit Philox word."""
+    if policy == "ess":
+        return int(round(value * 65536))
+    if policy == "freq":
+        return int(round(value * 2.0**32))   # > 2^32 is rejected by pf_init (PF_EINVAL)
+    return 0
+
+
 def _f32(a) -> np.ndarray:
     return np.ascontiguousarray(a, dtype=np.float32)
 
@@ -52,18 +65,25 @@ class ParticleFilter:
 
     ``n_filters=1`` with ``m > 1024`` (a multiple of 4096) is the paper's
     centralized filter (§VI, Fig. 9): one filter resampled
-    globally over all ``m`` particles (RWS; pf_central.cu).
+    globally over all ``m`` particles (RWS or Vose; pf_central.cu).
+
+    ``policy`` (reading R21, §IV): 'always' (default), 'ess'
+    (resample a sub-filter when its effective sample size falls below
+    ``policy_value`` x m) or 'freq' (each sub-filter resamples with
+    probability ``policy_value`` per step).
     """
 
     def __init__(self, mu0, sigma0, model: ArmModel | None = None, m: int = 256, n_filters: int = 4096,
                  t: int = 1, topo: str = "ring", resampler: str = "rws", seed: int = 0, rank: int = 0,
                  world: int = 1, torus_rows: int = 0, torus_cols: int = 0, device_inputs: bool = False,
-                 device: torch.device | int | None = None, stream: torch.cuda.Stream | None = None):
+                 device: torch.device | int | None = None, stream: torch.cuda.Stream | None = None,
+                 policy: str = "always", policy_value: float = 1.0):
         self.model = model or ArmModel()
         self.device = torch.device("cuda", torch.cuda.current_device() if device is None else
                                    (device if isinstance(device, int) else device.index or 0))
         self.cfg = B.pf_config(m, n_filters, t, TOPO[topo], torus_rows, torus_cols, RESAMPLER[resampler],
-                               seed, rank, world, B.PF_DEVICE_INPUTS if device_inputs else 0)
+                               seed, rank, world, B.PF_DEVICE_INPUTS if device_inputs else 0,
+                               POLICY[policy], _policy_param(policy, policy_value))
         self.m, self.n_filters, self.t, self.topo, self.resampler = m, n_filters, t, topo, resampler
         self.rank, self.world = rank, world
         self.d = self.model.d
