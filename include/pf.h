@@ -194,6 +194,25 @@ pf_status pf_step_batch(pf_handle* h, int32_t T, const float* zs, const float* u
  * PF_ESTATE before the first step. */
 pf_status pf_estimate(pf_handle* h, float* x_hat, float* logw, int64_t* idx);
 
+/* Weighted-average estimate of the last step's weighted set ("The
+ * reduction operator can compute the particle with the highest weight, a
+ * weighted average, or any other associative operator", §VI-D;
+ * reading R22): x_c = sum_p w_p x_cp / sum_p w_p with the integer weights
+ * w_p = floor(2^22 exp(l_p - L)) of F7, L = the best log-weight of the
+ * estimate record; numerators summed in double (each product exact),
+ * divided once.  x_mean: host float[d].  One extra read pass over the
+ * particle set; synchronizes.  world == 1 (else PF_ESTATE: use the two
+ * calls below); PF_ESTATE before the first step. */
+pf_status pf_estimate_mean(pf_handle* h, float* x_mean);
+
+/* Sharded filters (world > 1), after pf_reduce_records made L global: this
+ * shard's partial record, device double[d+1] = [sum w (uint64 bit pattern),
+ * sum w x_0, ..., sum w x_{d-1}] (stream-ordered, asynchronous), and the
+ * mean of `count` such records (device [count][d+1], e.g. an all-gather;
+ * summed in order) into host float[d] (synchronizes). */
+pf_status pf_mean_partial(pf_handle* h, double** partial_dev, int32_t* partial_doubles);
+pf_status pf_reduce_means(pf_handle* h, const double* partials_dev, int32_t count, float* x_mean);
+
 /* Device pointer to this shard's estimate record of the last step:
  * float[4 + d] = [key lo (u32 bits), key hi (u32 bits), logw, reserved, x[d]]
  * with key = (ordered(logw) << 32) | (0xffffffff - global index). */

@@ -142,6 +142,10 @@ orc_s_filter* orc_s_create(const orc_config* cfg, const orc_model* md, const flo
  * then sample + weight + estimate of step k.  z: n_joints+2, u: n_joints. */
 int orc_s_step(orc_s_filter* f, const float* z, const float* u);
 int orc_s_estimate(const orc_s_filter* f, float* x_hat, float* logw, int64_t* idx);
+/* Weighted-average estimate of the current set (R22; §VI-D). */
+int orc_s_estimate_mean(const orc_s_filter* f, float* x_mean);
+void orc_s_weighted_mean(const float* state, const float* logw, int64_t M, int32_t d, float* out);
+void orc_d_weighted_mean(const double* state, const double* logw, int64_t M, int32_t d, double* out);
 /* The weighted (pre-exchange) set of the current step; step 0 = prior. */
 int orc_s_get(const orc_s_filter* f, float* state, float* logw, int64_t* step);
 int orc_s_set(orc_s_filter* f, const float* state, const float* logw, int64_t step);
@@ -167,6 +171,7 @@ orc_d_filter* orc_d_create(const orc_config* cfg, const orc_model* md, const dou
                            const double* sigma0);
 int orc_d_step(orc_d_filter* f, const double* z, const double* u);
 int orc_d_estimate(const orc_d_filter* f, double* x_hat, double* logw, int64_t* idx);
+int orc_d_estimate_mean(const orc_d_filter* f, double* x_mean);
 int orc_d_get(const orc_d_filter* f, double* state, double* logw, int64_t* step);
 void orc_d_destroy(orc_d_filter* f);
 

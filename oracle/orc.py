@@ -84,6 +84,10 @@ def lib():
             "orc_d_sample_weight": (None, [P, C.c_uint64, C.c_int64, C.c_int64, P, P, P, C.c_int64, P, P]),
             "orc_rws_draw": (C.c_int32, [P, C.c_int32, C.c_uint32]),
             "orc_vose_build": (None, [P, C.c_int32, P, P]),
+            "orc_s_weighted_mean": (None, [P, P, C.c_int64, C.c_int32, P]),
+            "orc_d_weighted_mean": (None, [P, P, C.c_int64, C.c_int32, P]),
+            "orc_s_estimate_mean": (C.c_int, [P, P]),
+            "orc_d_estimate_mean": (C.c_int, [P, P]),
             "orc_should_resample": (C.c_int, [C.c_int32, C.c_uint64, P, C.c_int32, C.c_uint64, C.c_int64,
                                               C.c_int64]),
             "orc_vose_draw": (C.c_int32, [P, P, C.c_int32, C.c_uint64, C.c_uint32, C.c_uint32]),
@@ -251,6 +255,16 @@ def rws_draw(q, U: int) -> int:
     return lib().orc_rws_draw(_p(qq), len(qq), U)
 
 
+def weighted_mean(state, logw, fp64: bool = False) -> np.ndarray:
+    """R22: integer-weighted average of a weighted set (state [d][M], logw [M])."""
+    conv = _f64 if fp64 else _f32
+    st, lw = conv(state), conv(logw)
+    d, M = st.shape
+    out = np.zeros(d, st.dtype)
+    (lib().orc_d_weighted_mean if fp64 else lib().orc_s_weighted_mean)(_p(st), _p(lw), M, d, _p(out))
+    return out
+
+
 def should_resample(policy: str, param: int, q, seed: int, n: int, k: int) -> bool:
     qq = _u32(q)
     return bool(lib().orc_should_resample(POLICY[policy], param, _p(qq), len(qq), seed, n, k))
@@ -368,7 +382,7 @@ class Filter:
         self.M = cfg.m * cfg.n_filters
         L = lib()
         pre = "orc_d_" if fp64 else "orc_s_"
-        self._fn = {n: getattr(L, pre + n) for n in ("create", "step", "estimate", "get", "destroy")}
+        self._fn = {n: getattr(L, pre + n) for n in ("create", "step", "estimate", "estimate_mean", "get", "destroy")}
         if not fp64:
             self._fn["set"] = L.orc_s_set
             self._fn["trace"] = L.orc_s_trace
@@ -398,6 +412,13 @@ class Filter:
         if rc:
             raise RuntimeError("no estimate before the first step")
         return x, w.value, idx.value
+
+    def estimate_mean(self) -> np.ndarray:
+        """R22: the weighted-average estimate of the current set."""
+        x = np.zeros(self.d, np.float64 if self.fp64 else np.float32)
+        if self._fn["estimate_mean"](self._h, _p(x)):
+            raise RuntimeError("no estimate before the first step")
+        return x
 
     def get(self):
         dt = np.float64 if self.fp64 else np.float32

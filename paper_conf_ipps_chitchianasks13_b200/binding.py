@@ -24,7 +24,8 @@ ENTRY_POINTS = [
     "pf_query_sizes", "pf_init", "pf_step", "pf_step_batch", "pf_estimate", "pf_record_ptr",
     "pf_reduce_records", "pf_reduce_pool", "pf_get_shard", "pf_get_particles", "pf_set_particles", "pf_debug_sample_weight",
     "pf_debug_resample", "pf_debug_exchange", "pf_set_trace", "pf_get_trace", "pf_destroy", "pf_strerror",
-    "pf_last_error", "pf_supported", "pf_debug_math", "pf_debug_check_sqrt",
+    "pf_last_error", "pf_supported", "pf_debug_math", "pf_debug_check_sqrt", "pf_estimate_mean", "pf_mean_partial",
+    "pf_reduce_means",
 ]
 PF_MATH = {"sin": 0, "cos": 1, "log": 2, "expq": 3, "sqrt": 4, "sincos2pi": 5, "normal_pair": 6, "philox": 7}
 
@@ -79,6 +80,9 @@ def lib() -> C.CDLL:
             "pf_step_batch": [P, I32, P, P, P],
             "pf_estimate": [P, P, P, P],
             "pf_record_ptr": [P, P, P],
+            "pf_estimate_mean": [P, P],
+            "pf_mean_partial": [P, P, P],
+            "pf_reduce_means": [P, P, I32, P],
             "pf_reduce_records": [P, P, I32],
             "pf_reduce_pool": [P],
             "pf_get_shard": [P, P],
@@ -150,6 +154,20 @@ def pf_estimate(h, x_hat) -> tuple[float, int]:
     lw, idx = C.c_float(), C.c_int64()
     check(lib().pf_estimate(h, _ptr(x_hat), C.byref(lw), C.byref(idx)), "pf_estimate")
     return lw.value, idx.value
+
+
+def pf_estimate_mean(h, x_mean) -> None:
+    check(lib().pf_estimate_mean(h, _ptr(x_mean)), "pf_estimate_mean")
+
+
+def pf_mean_partial(h) -> tuple[int, int]:
+    p, n = C.c_void_p(), C.c_int32()
+    check(lib().pf_mean_partial(h, C.byref(p), C.byref(n)), "pf_mean_partial")
+    return p.value, n.value
+
+
+def pf_reduce_means(h, partials_dev, count: int, x_mean) -> None:
+    check(lib().pf_reduce_means(h, _ptr(partials_dev), count, _ptr(x_mean)), "pf_reduce_means")
 
 
 def pf_record_ptr(h) -> tuple[int, int]:

@@ -13,6 +13,7 @@
 
 #include "../../include/pf.h"
 #include "pf_central.h"
+#include "pf_mean.h"
 #include "pf_kernels.cuh"
 #include "pf_registry.h"
 
@@ -30,7 +31,8 @@ constexpr size_t kOffRecord = 64;     // float[4 + d]  (d <= 32 -> 144 B)
 constexpr size_t kOffInputs = 256;    // float[64]: z at 0, u at 32
 constexpr size_t kOffMu0 = 512;       // float[64]
 constexpr size_t kOffSigma0 = 768;    // float[64]
-constexpr size_t kScratchBytes = 1024;
+constexpr size_t kOffMean = 1024;     // double[kMeanGrid + 1][33]: weighted-mean partials + summed record
+constexpr size_t kScratchBytes = kOffMean + sizeof(double) * (pf::kMeanGrid + 1) * 33;
 
 struct Table {
   const pf::KernelEntry* e;
@@ -196,7 +198,7 @@ struct pf_handle {
   bool trace;
   long long* d_src;
   int* d_anc;
-  float* rec_host;     // mapped pinned host copy of the estimate record (written by the kernels)
+  float* rec_host;     // mapped pinned host floats: [0, 4+d) estimate record, [48, 48+d) weighted mean
   float* rec_host_dev; // its device alias
   float* d_reduce_tmp;
 };
@@ -491,7 +493,7 @@ pf_status pf_init(const pf_config* cfg, const pf_model_params* model, const pf_b
   }
   if (e == cudaSuccess && bps < 1) e = cudaErrorInvalidConfiguration;
   if (e == cudaSuccess)
-    e = cudaHostAlloc(reinterpret_cast<void**>(&h->rec_host), sizeof(float) * 64, cudaHostAllocMapped);
+    e = cudaHostAlloc(reinterpret_cast<void**>(&h->rec_host), sizeof(float) * 128, cudaHostAllocMapped);
   if (e == cudaSuccess) e = cudaHostGetDevicePointer(reinterpret_cast<void**>(&h->rec_host_dev), h->rec_host, 0);
   if (e != cudaSuccess) {
     pf_destroy(h);
@@ -630,6 +632,62 @@ pf_status pf_estimate(pf_handle* h, float* x_hat, float* logw, int64_t* idx) {
   std::memcpy(x_hat, rec + 4, sizeof(float) * h->g.d);
   if (logw) *logw = rec[2];
   if (idx) *idx = static_cast<int64_t>(0xFFFFFFFFu - lo);
+  return PF_OK;
+}
+
+// ---- weighted-average estimate (R22) -------------------------------------
+static double* mean_scratch(pf_handle* h) { return reinterpret_cast<double*>(h->scratch + kOffMean); }
+
+static pf_status mean_partials_launch(pf_handle* h) {
+  pf::MeanParams mp;
+  mp.parts = set_of_step(h, h->step);
+  mp.n_blocks = h->g.central ? 1 : h->g.n_local;
+  mp.m = h->g.central ? static_cast<int>(h->g.M_local) : h->g.m;
+  mp.d = h->g.d;
+  mp.row = h->g.ROW;
+  mp.record = record(h);
+  mp.partials = mean_scratch(h);
+  return sticky(h, pf::mean_partials(mp, h->stream));
+}
+
+pf_status pf_estimate_mean(pf_handle* h, float* x_mean) {
+  if (!h || !x_mean) return PF_EINVAL;
+  if (h->err != PF_OK) return h->err;
+  if (h->step < 1) return PF_ESTATE;
+  if (h->cfg.world != 1) return PF_ESTATE;
+  pf_status st = mean_partials_launch(h);
+  if (st != PF_OK) return st;
+  float* out = h->rec_host_dev + 48;   // mapped pinned host floats [48, 48 + d) (record uses [0, 4 + d))
+  st = sticky(h, pf::mean_final(mean_scratch(h), pf::kMeanGrid, h->g.d, nullptr, nullptr, out, h->stream));
+  if (st != PF_OK) return st;
+  cudaError_t e = cudaStreamSynchronize(h->stream);
+  if (e != cudaSuccess) return sticky(h, e);
+  std::memcpy(x_mean, const_cast<const float*>(h->rec_host) + 48, sizeof(float) * h->g.d);
+  return PF_OK;
+}
+
+pf_status pf_mean_partial(pf_handle* h, double** partial_dev, int32_t* partial_doubles) {
+  if (!h || !partial_dev) return PF_EINVAL;
+  if (h->err != PF_OK) return h->err;
+  if (h->step < 1) return PF_ESTATE;
+  pf_status st = mean_partials_launch(h);
+  if (st != PF_OK) return st;
+  double* rec = mean_scratch(h) + static_cast<long long>(pf::kMeanGrid) * 33;
+  st = sticky(h, pf::mean_final(mean_scratch(h), pf::kMeanGrid, h->g.d, rec, nullptr, nullptr, h->stream));
+  *partial_dev = rec;
+  if (partial_doubles) *partial_doubles = h->g.d + 1;
+  return st;
+}
+
+pf_status pf_reduce_means(pf_handle* h, const double* partials_dev, int32_t count, float* x_mean) {
+  if (!h || !partials_dev || count < 1 || !x_mean) return PF_EINVAL;
+  if (h->err != PF_OK) return h->err;
+  float* out = h->rec_host_dev + 48;
+  pf_status st = sticky(h, pf::mean_final(partials_dev, count, h->g.d, nullptr, nullptr, out, h->stream));
+  if (st != PF_OK) return st;
+  cudaError_t e = cudaStreamSynchronize(h->stream);
+  if (e != cudaSuccess) return sticky(h, e);
+  std::memcpy(x_mean, const_cast<const float*>(h->rec_host) + 48, sizeof(float) * h->g.d);
   return PF_OK;
 }
 

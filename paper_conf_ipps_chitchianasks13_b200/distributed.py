@@ -152,3 +152,14 @@ class DistributedFilter:
 
     def estimate(self):
         return self.pf.estimate()
+
+    def estimate_mean(self):
+        """Weighted-average estimate (R22) of the whole sharded filter: every
+        rank's partial record (with the global L of the reduced record) is
+        all-gathered and summed in rank order."""
+        if self.world == 1:
+            return self.pf.estimate_mean()
+        part = self.pf.mean_partial()
+        gathered = torch.empty(self.world, part.numel(), dtype=torch.float64, device=part.device)
+        dist.all_gather_into_tensor(gathered, part.contiguous(), group=self.group)
+        return self.pf.reduce_means(gathered)

@@ -145,6 +145,24 @@ class ParticleFilter:
         lw, idx = B.pf_estimate(self.h, self._xhat)
         return self._xhat.copy(), lw, idx
 
+    def estimate_mean(self) -> np.ndarray:
+        """Weighted-average estimate x [d] of the last step's set (R22; §VI-D)."""
+        x = np.zeros(self.d, np.float32)
+        B.pf_estimate_mean(self.h, x)
+        return x
+
+    def mean_partial(self) -> torch.Tensor:
+        """World > 1: this shard's partial record (device float64 [d+1]; slot 0 = uint64 bits)."""
+        ptr, n = B.pf_mean_partial(self.h)
+        off = ptr - self._scratch.data_ptr()
+        return self._scratch[off: off + 8 * n].view(torch.float64)
+
+    def reduce_means(self, partials: torch.Tensor) -> np.ndarray:
+        """Mean of gathered partial records [count][d+1] (device float64)."""
+        x = np.zeros(self.d, np.float32)
+        B.pf_reduce_means(self.h, partials.data_ptr(), partials.shape[0], x)
+        return x
+
     def reduce_records(self, records: torch.Tensor) -> None:
         B.pf_reduce_records(self.h, records.data_ptr(), records.shape[0])
 

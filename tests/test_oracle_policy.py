@@ -126,3 +126,53 @@ def test_freq_mixed_steps(orc, W):
                 np.testing.assert_array_equal(anc[sl], np.arange(16))
                 np.testing.assert_array_equal(w1[sl], (w0[sl] - w0[sl].max()).astype(np.float32) + ll)
     assert kinds == {True, False}
+
+
+# ---- weighted-average estimate (R22; §VI-D "a weighted average") ----
+
+def test_weighted_mean_equal_weights_is_the_mean(orc):
+    rng = np.random.default_rng(3)
+    x = rng.normal(0, 2, (6, 1000)).astype(np.float32)
+    got = orc.weighted_mean(x, np.full(1000, -3.25, np.float32))
+    np.testing.assert_allclose(got, x.astype(np.float64).mean(axis=1), rtol=1e-6, atol=1e-7)
+
+
+def test_weighted_mean_dominant_particle(orc):
+    # every other weight below e^-16 of the best is dropped (F7): exactly that particle
+    rng = np.random.default_rng(4)
+    x = rng.normal(0, 1, (5, 300)).astype(np.float32)
+    lw = rng.uniform(-80, -20, 300).astype(np.float32)
+    lw[123] = -1.0
+    np.testing.assert_array_equal(orc.weighted_mean(x, lw), x[:, 123])
+
+
+def test_weighted_mean_vs_exact_weights(orc):
+    # against the plain definition sum w x / sum w with float64 weights exp(l - L):
+    # the 2^-22 quantisation of the integer weights bounds the difference
+    rng = np.random.default_rng(5)
+    for M in (7, 256, 4096):
+        x = rng.normal(0, 1, (9, M)).astype(np.float32)
+        lw = (-rng.exponential(2.0, M)).astype(np.float32)
+        w = np.exp(lw.astype(np.float64) - lw.max())
+        ref = (x.astype(np.float64) * w).sum(axis=1) / w.sum()
+        got = orc.weighted_mean(x, lw)
+        np.testing.assert_allclose(got, ref, rtol=0, atol=4 * M * 2.0**-22 / w.sum() * np.abs(x).max() + 1e-6)
+        got64 = orc.weighted_mean(x, lw, fp64=True)
+        np.testing.assert_allclose(got64, ref, rtol=0, atol=4 * M * 2.0**-22 / w.sum() * np.abs(x).max() + 1e-9)
+
+
+def test_filter_mean_estimate_tracks(orc, W):
+    # the weighted average of the filter's own set, after it converged, lies
+    # near its max-weight estimate and near the true object position
+    nj, T = 2, 40
+    tr = W.make_trajectory(nj, T, 0)
+    f = orc.Filter(orc.Config(m=64, n_filters=16, t=1, topo="ring", seed=2), orc.Model(n_joints=nj),
+                   tr["mu0"], tr["sigma0"])
+    err = []
+    for k in range(1, T + 1):
+        f.step(tr["Z"][k], tr["U"][k - 1])
+        xm = f.estimate_mean()
+        s, w, _ = f.get()
+        np.testing.assert_array_equal(xm, orc.weighted_mean(s, w))
+        err.append(np.hypot(*(xm[nj:nj + 2] - tr["X"][k][nj:nj + 2])))
+    assert np.sqrt(np.mean(np.square(err[10:]))) < 0.25
