@@ -275,21 +275,33 @@ def run_ours(a) -> None:
         pass
     peak = peaks.get("hbm_gbs", 6650.0)
     achieved = bytes_launch / (ms_step * 1e-3) / 1e9
-    traffic = None
+    traffic, instr = None, None
     try:
         prof = json.load(open(os.path.join(ROOT, "profiles", "ncu_summary.json")))
         traffic = prof.get("C2", {}).get("dram_bytes_per_launch")
+        instr = prof.get("C2", {}).get("lane_instr_per_particle")
     except Exception:
         pass
     roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
                 "traffic": traffic, "kernel": "pf_step_kernel", "bytes_per_launch": bytes_launch,
                 "peak_source": "MEASURED_PEAKS.json hbm_gbs" if "hbm_gbs" in peaks else "fallback 6.65 TB/s",
-                "note": "issue-bound: see DESIGN.md §6 for the instruction roofline"}
+                "note": "issue-bound: see roofline_issue and DESIGN.md §6"}
+    # the binding roofline: instruction issue (148 SMs x 4 schedulers x 32 lanes
+    # per clock at the sampled SM clock); executed lane-instructions per
+    # particle-step from the committed ncu capture of this kernel at C2
+    roofline_issue = None
+    if instr:
+        mhz = clocks.get("sm_mhz") or 1965
+        peak_i = 148 * 4 * 32 * mhz * 1e6 / 1e12
+        ach_i = instr * PARTICLES_PER_GPU / (ms_step * 1e-3) / 1e12
+        roofline_issue = {"bound": "alu", "achieved": ach_i, "peak": peak_i, "unit": "T lane-instr/s",
+                          "frac": ach_i / peak_i, "instr_per_particle": instr,
+                          "source": "profiles/ncu_summary.json C2 smsp__inst_executed x 32 / particles"}
 
     line = {"metric": METRIC, "value": value, "unit": "particle-steps/s", "n_gpus": world, "steps": K,
             "warmup": Wm, "ms_per_step": ms_step, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
             "dtype": "f32", "data": DATA, "config": _config(world), "estimates_per_s": steps_per_s,
-            "roofline": roofline,
+            "roofline": roofline, "roofline_issue": roofline_issue,
             "e2e": {"value": e2e_value, "unit": "particle-steps/s", "estimates_per_s": 1e3 / e2e_ms,
                     "ms_per_step": e2e_ms, "h2d_bytes_per_step": 4 * (NJ + 2 + NJ),
                     "d2h_bytes_per_step": 4 * (4 + D)},

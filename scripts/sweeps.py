@@ -10,10 +10,10 @@ from paper_conf_ipps_chitchianasks13_b200 import filter as F, workload as W
 flush = torch.empty(512 << 20, dtype=torch.uint8, device="cuda")
 
 
-def run(tag, nj, m, N, res="rws", topo="ring", t=1, steps=20, warm=3):
+def run(tag, nj, m, N, res="rws", topo="ring", t=1, steps=20, warm=3, policy="always", value=1.0):
     tr = W.make_trajectory(nj, steps + warm + 4, 0)
     g = F.ParticleFilter(tr["mu0"], tr["sigma0"], F.ArmModel(n_joints=nj), m=m, n_filters=N, t=t, topo=topo,
-                         resampler=res, seed=7, device_inputs=True)
+                         resampler=res, seed=7, device_inputs=True, policy=policy, policy_value=value)
     zs = torch.tensor(tr["Z"][1:], device="cuda")
     us = torch.tensor(tr["U"][:-1], device="cuda")
     for k in range(warm):
@@ -30,14 +30,14 @@ def run(tag, nj, m, N, res="rws", topo="ring", t=1, steps=20, warm=3):
     M, d = m * N, nj + 4
     bytes_ = M * 8 * (d + 1)
     out = {"sweep": tag, "n_joints": nj, "d": d, "m": m, "N": N, "particles": M, "resampler": res, "topo": topo,
-           "t": t, "us_per_step": ms * 1e3, "estimates_per_s": 1e3 / ms, "particle_steps_per_s": M / (ms * 1e-3),
+           "t": t, "policy": policy, "policy_value": value, "us_per_step": ms * 1e3, "estimates_per_s": 1e3 / ms, "particle_steps_per_s": M / (ms * 1e-3),
            "hbm_gbs_algorithmic": bytes_ / (ms * 1e-3) / 1e9}
     print(json.dumps(out), flush=True)
     g.close()
 
 
 if __name__ == "__main__":
-    which = sys.argv[1:] or ["count", "m", "t", "dim", "res"]
+    which = sys.argv[1:] or ["count", "m", "t", "dim", "res", "central", "policy"]
     if "count" in which:   # Fig.3 / Fig.4b analogue: particle count (m = 256, d = 9)
         for N in [4, 16, 64, 256, 1024, 4096, 16384, 65536, 262144, 390625]:
             run("count", 5, 256, N, steps=10 if N > 100000 else 20)
@@ -55,3 +55,10 @@ if __name__ == "__main__":
         for nj, N in [(5, 4096), (5, 65536), (28, 65536)]:
             for res in ["rws", "vose"]:
                 run("res", nj, 256, N, res=res)
+    if "central" in which:  # Fig.5 centralized curves / Fig.9: one filter of M particles (NEXT-2)
+        for M in [1 << 14, 1 << 16, 1 << 18, 1 << 20]:
+            for res in ["rws", "vose"]:
+                run("central", 5, M, 1, res=res, topo="none", t=0)
+    if "policy" in which:   # §IV conditional resampling (NEXT-4) at C2
+        for policy, value in [("always", 1.0), ("ess", 0.05), ("freq", 0.5), ("freq", 0.1)]:
+            run("policy", 5, 256, 4096, policy=policy, value=value)
