@@ -282,6 +282,80 @@ __device__ __forceinline__ X slot_scan_incl(const X (&val)[C::P], X (&out)[C::P]
   }
 }
 
+// P contiguous elements <-> registers with the widest shared-memory vectors
+template <typename X, int P>
+__device__ __forceinline__ void vload(const X* src, X (&v)[P]) {
+  constexpr int B = P * static_cast<int>(sizeof(X));
+  if constexpr (B % 16 == 0) {
+#pragma unroll
+    for (int i = 0; i < B / 16; ++i) reinterpret_cast<uint4*>(v)[i] = reinterpret_cast<const uint4*>(src)[i];
+  } else if constexpr (B % 8 == 0) {
+#pragma unroll
+    for (int i = 0; i < B / 8; ++i) reinterpret_cast<uint2*>(v)[i] = reinterpret_cast<const uint2*>(src)[i];
+  } else {
+#pragma unroll
+    for (int i = 0; i < P; ++i) v[i] = src[i];
+  }
+}
+template <typename X, int P>
+__device__ __forceinline__ void vstore(X* dst, const X (&v)[P]) {
+  constexpr int B = P * static_cast<int>(sizeof(X));
+  if constexpr (B % 16 == 0) {
+#pragma unroll
+    for (int i = 0; i < B / 16; ++i) reinterpret_cast<uint4*>(dst)[i] = reinterpret_cast<const uint4*>(v)[i];
+  } else if constexpr (B % 8 == 0) {
+#pragma unroll
+    for (int i = 0; i < B / 8; ++i) reinterpret_cast<uint2*>(dst)[i] = reinterpret_cast<const uint2*>(v)[i];
+  } else {
+#pragma unroll
+    for (int i = 0; i < P; ++i) dst[i] = v[i];
+  }
+}
+
+// Slot-order inclusive prefix through shared memory: the strided per-thread
+// values are transposed (buf[slot]), thread t scans the P contiguous slots
+// [tP, tP + P) serially, ONE warp shuffle scan of the per-thread totals (plus
+// one cross-warp level) replaces the P shuffle scans of slot_scan_incl, and
+// buf[s] ends up holding the inclusive prefix of every slot s (slot order).
+// Returns the group total.  Group barriers: 2 (+1 when GW > 1).
+template <class C, typename X>
+__device__ __forceinline__ X slot_scan_smem(const X (&val)[C::P], X* buf, GroupCtx& G) {
+  constexpr int P = C::P, GW = C::GW;
+#pragma unroll
+  for (int j = 0; j < P; ++j) buf[C::slot(G.t, j)] = val[j];
+  gsync<GW>(G.g);
+  X v[P];
+  vload<X, P>(buf + G.t * P, v);
+#pragma unroll
+  for (int j = 1; j < P; ++j) v[j] += v[j - 1];
+  const X tot = v[P - 1];
+  const X inc = warp_incl_scan<X>(tot, G.lane);
+  X off = inc - tot;
+  X total;
+  if constexpr (GW == 1) {
+    total = __shfl_sync(0xFFFFFFFFu, inc, 31);
+  } else {
+    X* r = reinterpret_cast<X*>(G.red + G.rb * 32);
+    G.rb ^= 1;
+    if (G.lane == 31) r[G.wig] = inc;
+    gsync<GW>(G.g);
+    X before = 0;
+    total = 0;
+#pragma unroll
+    for (int w = 0; w < GW; ++w) {
+      const X x = r[w];
+      if (w < G.wig) before += x;
+      total += x;
+    }
+    off += before;
+  }
+#pragma unroll
+  for (int j = 0; j < P; ++j) v[j] += off;
+  vstore<X, P>(buf + G.t * P, v);
+  gsync<GW>(G.g);
+  return total;
+}
+
 // first index i in [0, n) with a[i] >= x
 __device__ __forceinline__ int lower_bound_u64(const u64* a, int n, u64 x) {
   int lo = 0;
@@ -331,14 +405,11 @@ __device__ __forceinline__ void resample_group(const uint32_t (&q)[C::P], const 
     // Roulette Wheel Selection (§VI-F): C = inclusive sums of q
     // in slot order, c = floor(U Q / 2^32), ancestor = first j with C_j > c.
     using X = typename std::conditional<C::SCAN32, uint32_t, u64>::type;
-    X val[P], inc[P];
+    X val[P];
 #pragma unroll
     for (int j = 0; j < P; ++j) val[j] = q[j];
-    const X Q = slot_scan_incl<C, X>(val, inc, G);
     X* Cs = reinterpret_cast<X*>(S.scan);
-#pragma unroll
-    for (int j = 0; j < P; ++j) Cs[C::slot(G.t, j)] = inc[j];
-    gsync<C::GW>(G.g);
+    const X Q = slot_scan_smem<C, X>(val, Cs, G);   // Cs[s] = inclusive sum of slot s
 #pragma unroll
     for (int j = 0; j < P; ++j) {
       const X c = static_cast<X>((static_cast<u64>(ua[j]) * Q) >> 32);
@@ -355,57 +426,73 @@ __device__ __forceinline__ void resample_group(const uint32_t (&q)[C::P], const 
     // Two slot-order scans: the weights (-> Q and the prefix of a = M q), and
     // the deficits over L with the count of L packed above bit 48 (D < 2^42).
     // E follows from sum_{j'<=j} (a_j' - Q) = E_j - D_j.
-    u64 val[P], qinc[P];
+    // Only the two inclusive scans stay live per slot (register budget); the
+    // per-slot class, deficit, counts and E are recomputed from them.
+    u64 qinc[P], pinc[P];
+    u64 Qg, ptot;
+    {
+      u64 val[P];
 #pragma unroll
-    for (int j = 0; j < P; ++j) val[j] = q[j];
-    const u64 Q = slot_scan_incl<C, u64>(val, qinc, G);
-    u64 a[P];
-    bool small[P];
-    u64 packed[P], pinc[P], cnt[P], def[P], Dinc[P], Einc[P];
+      for (int j = 0; j < P; ++j) val[j] = q[j];
+      Qg = slot_scan_smem<C, u64>(val, S.scan, G);
 #pragma unroll
-    for (int j = 0; j < P; ++j) {
-      a[j] = static_cast<u64>(M) * q[j];
-      small[j] = a[j] < Q;
-      def[j] = small[j] ? Q - a[j] : 0ull;
-      packed[j] = def[j] + (small[j] ? (1ull << 48) : 0ull);
+      for (int j = 0; j < P; ++j) qinc[j] = S.scan[C::slot(G.t, j)];
     }
-    const u64 ptot = slot_scan_incl<C, u64>(packed, pinc, G);
+    {
+      u64 packed[P];
+#pragma unroll
+      for (int j = 0; j < P; ++j) {
+        const u64 a = static_cast<u64>(M) * q[j];
+        packed[j] = a < Qg ? (Qg - a) + (1ull << 48) : 0ull;
+      }
+      ptot = slot_scan_smem<C, u64>(packed, S.prob, G);
+#pragma unroll
+      for (int j = 0; j < P; ++j) pinc[j] = S.prob[C::slot(G.t, j)];
+    }
+    // (every thread read qinc before passing scan 2's barriers: S.scan is free)
     const int nL = static_cast<int>(ptot >> 48);
     const u64 Dtot = ptot & ((1ull << 48) - 1);
-#pragma unroll
-    for (int j = 0; j < P; ++j) {
-      cnt[j] = pinc[j] >> 48;
-      Dinc[j] = pinc[j] & ((1ull << 48) - 1);
+    auto cls = [&](int j, bool& small, u64& a, u64& Dinc, u64& Einc, int& ls) {
+      a = static_cast<u64>(M) * q[j];
+      small = a < Qg;
+      Dinc = pinc[j] & ((1ull << 48) - 1);
+      ls = static_cast<int>(pinc[j] >> 48) - (small ? 1 : 0);   // smalls before the slot
       const u64 slot1 = static_cast<u64>(C::slot(G.t, j)) + 1;
-      Einc[j] = Dinc[j] + static_cast<u64>(M) * qinc[j] - slot1 * Q;
-    }
+      Einc = Dinc + static_cast<u64>(M) * qinc[j] - slot1 * Qg;
+    };
 #pragma unroll
     for (int j = 0; j < P; ++j) {
+      bool small;
+      u64 a, Dinc, Einc;
+      int ls;
+      cls(j, small, a, Dinc, Einc, ls);
       const int s = C::slot(G.t, j);
-      const int ls = static_cast<int>(cnt[j]) - (small[j] ? 1 : 0);   // smalls before s
-      if (small[j]) {
+      if (small) {
         S.lists[ls] = s;
-        S.scan[ls] = Dinc[j];
+        S.scan[ls] = Dinc;
       } else {
         S.lists[nL + (s - ls)] = s;
-        S.scan[nL + (s - ls)] = Einc[j];
+        S.scan[nL + (s - ls)] = Einc;
       }
     }
     gsync<C::GW>(G.g);
 #pragma unroll
     for (int j = 0; j < P; ++j) {
+      bool small;
+      u64 a, Dinc, Einc;
+      int ls;
+      cls(j, small, a, Dinc, Einc, ls);
       const int s = C::slot(G.t, j);
-      const int ls = static_cast<int>(cnt[j]) - (small[j] ? 1 : 0);
       u64 pr;
       int al;
-      if (small[j]) {
-        pr = a[j];
-        al = S.lists[nL + lower_bound_u64(S.scan + nL, M - nL, Dinc[j] - def[j])];
-      } else if (Einc[j] < Dtot) {
-        pr = Q + Einc[j] - S.scan[upper_bound_u64(S.scan, nL, Einc[j])];
+      if (small) {
+        pr = a;
+        al = S.lists[nL + lower_bound_u64(S.scan + nL, M - nL, Dinc - (Qg - a))];
+      } else if (Einc < Dtot) {
+        pr = Qg + Einc - S.scan[upper_bound_u64(S.scan, nL, Einc)];
         al = S.lists[nL + (s - ls) + 1];
       } else {
-        pr = Q;
+        pr = Qg;
         al = s;
       }
       S.prob[s] = pr;
@@ -415,11 +502,12 @@ __device__ __forceinline__ void resample_group(const uint32_t (&q)[C::P], const 
         alias_out[s] = al;
       }
     }
+    const u64 Q2 = Qg;
     gsync<C::GW>(G.g);
 #pragma unroll
     for (int j = 0; j < P; ++j) {
       const int b = static_cast<int>((static_cast<u64>(ua[j]) * M) >> 32);
-      const u64 c = (static_cast<u64>(ub[j]) * Q) >> 32;
+      const u64 c = (static_cast<u64>(ub[j]) * Q2) >> 32;
       anc[j] = c < S.prob[b] ? b : S.alias[b];
     }
   }
