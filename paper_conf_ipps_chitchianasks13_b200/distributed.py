@@ -160,6 +160,6 @@ class DistributedFilter:
         if self.world == 1:
             return self.pf.estimate_mean()
         part = self.pf.mean_partial()
-        gathered = torch.empty(self.world, part.numel(), dtype=torch.float64, device=part.device)
+        gathered = torch.empty(self.world * part.numel(), dtype=torch.float64, device=part.device)
         dist.all_gather_into_tensor(gathered, part.contiguous(), group=self.group)
-        return self.pf.reduce_means(gathered)
+        return self.pf.reduce_means(gathered.view(self.world, part.numel()))

@@ -116,3 +116,53 @@ def test_plan_shapes():
     assert len(p) == 8 and all(t.nrows == 8 for t in p)
     assert Dd.shard_geometry("torus", 64, 4, 3) == (48, 16, 32)
     assert Dd.shard_geometry("ring", 64, 4, 1) == (16, 16, 18)
+
+
+class _FakeShard:
+    """Host stand-in for a ParticleFilter shard: the partial record of R22
+    (pf_mean_partial) computed on the host from the global L."""
+
+    def __init__(self, state, logw, L, rank, world, orc):
+        self.state, self.logw, self.L, self.orc = state, logw, L, orc
+        self.rank, self.world = rank, world
+
+    def mean_partial(self):
+        q = np.array([self.orc.s_expq(float(v - self.L)) for v in self.logw], np.float64)
+        S = (self.state.astype(np.float64) * q).sum(axis=1)
+        Q = int(q.sum())
+        return torch.tensor(np.concatenate([np.array([Q], np.int64).view(np.float64), S]))
+
+    def reduce_means(self, parts):
+        p = parts.numpy()
+        Q = int(p[:, 0].copy().view(np.int64).sum())
+        return (p[:, 1:].sum(axis=0) / Q).astype(np.float32)
+
+
+def _mean_worker(rank, world, port, ret):
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        from oracle import orc
+        orc.build()
+        rng = np.random.default_rng(3)
+        state = rng.normal(0, 1, (6, 40 * world)).astype(np.float32)
+        logw = (-rng.exponential(3.0, 40 * world)).astype(np.float32)
+        sl = slice(rank * 40, (rank + 1) * 40)
+        df = Dd.DistributedFilter.__new__(Dd.DistributedFilter)
+        df.pf, df.group, df.rank, df.world = _FakeShard(state[:, sl], logw[sl], logw.max(), rank, world, orc), None, \
+            rank, world
+        got = df.estimate_mean()
+        np.testing.assert_allclose(got, orc.weighted_mean(state, logw), rtol=1e-6, atol=1e-7)
+        ret[rank] = True
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world", [2, 3])
+def test_mean_protocol_gloo(world):
+    # R22 across ranks: every rank's partial record (global L) all-gathered in
+    # rank order and reduced = the weighted mean of the whole set
+    ctx = mp.get_context("spawn")
+    ret = ctx.Manager().dict()
+    mp.start_processes(_mean_worker, args=(world, _free_port(), ret), nprocs=world, join=True, start_method="spawn")
+    assert len(ret) == world
