@@ -18,6 +18,7 @@ const KernelEntry kEntriesNJ5[] = {
     PF_ENTRY(5, 256, 0, 4, 2, 1, 1, 4), PF_ENTRY(5, 256, 0, 1, 8, 1, 1, 4), PF_ENTRY(5, 256, 0, 2, 4, 1, 4, 2),
     PF_ENTRY(5, 256, 0, 2, 3, 1, 4, 3),
     PF_ENTRY(5, 256, 1, 2, 4, 1, 1, 4), PF_ENTRY(5, 256, 1, 2, 3, 1, 1, 4),
+    PF_ENTRY(5, 256, 0, 2, 3, 2, 1, 3), PF_ENTRY(5, 256, 0, 2, 4, 2, 1, 2), PF_ENTRY(5, 256, 0, 2, 2, 2, 1, 4),
 };
 const int kNumEntriesNJ5 = sizeof(kEntriesNJ5) / sizeof(kEntriesNJ5[0]);
 }  // namespace pf

@@ -1092,12 +1092,19 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
               float* e = P.mb_cur + (n * P.tt + jb) * E;
               e[0] = lnew[j];
               e[1] = __uint_as_float(pbase + bslot);
-              // own global write (same thread: program order) or the loaded set
-              const float* src = do_sample ? gblk + bslot : xs + bslot;
-#pragma unroll 4
-              for (int c = 0; c < D; ++c) e[2 + c] = src[c * M];
             }
             if (jb == 0) atomicMax(P.key_cur, best);
+          }
+        }
+        if (jb < P.t && G.wig == 0) {
+          // the state of the best particle, one component per lane (one L2
+          // round trip): the owner's global stores of the sample loop are
+          // ordered before these loads by the group barrier in gmax (GW > 1)
+          // or the warp barrier (GW == 1); without sampling: the loaded set
+          if constexpr (GW == 1) __syncwarp();
+          if (G.lane < D) {
+            const float* src = do_sample ? gblk + bslot : xs + bslot;
+            P.mb_cur[(n * P.tt + jb) * E + 2 + G.lane] = src[G.lane * M];
           }
         }
       }
@@ -1107,9 +1114,11 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
 
   // ---- a5: the last CTA to finish copies the winning particle (R6)
   __shared__ unsigned int s_last;
-  __threadfence();
   __syncthreads();
   if (threadIdx.x == 0) {
+    // the CTA barrier orders every thread's writes (mailbox rows, key) before
+    // thread 0's cumulative gpu-scope fence and the completion count
+    __threadfence();
     const unsigned int prev = atomicAdd(P.counter, 1u);
     s_last = (prev == gridDim.x - 1) ? 1u : 0u;
   }

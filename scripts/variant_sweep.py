@@ -1,7 +1,8 @@
 """Dev tool: time every compiled mapping (PF_VARIANT=i) of one (nj, m, res) at given N.
-usage: variant_sweep.py nj m res N1,N2,... nvariants"""
+usage: variant_sweep.py nj m res N1,N2,... nvariants | v1,v2,... (-1 = auto)"""
 import os, subprocess, sys
-nj, m, res, Ns, nv = sys.argv[1], sys.argv[2], sys.argv[3], sys.argv[4].split(","), int(sys.argv[5])
+nj, m, res, Ns = sys.argv[1], sys.argv[2], sys.argv[3], sys.argv[4].split(",")
+vs = [int(v) for v in sys.argv[5].split(",")] if "," in sys.argv[5] else list(range(-1, int(sys.argv[5])))
 code = r'''
 import sys, os; sys.path.insert(0, os.getcwd())
 import torch
@@ -16,7 +17,7 @@ e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=Tr
 e0.record(g.stream); g.step_batch(zs[5:5+T], us[5:5+T]); e1.record(g.stream); torch.cuda.synchronize()
 print(f"{e0.elapsed_time(e1) / T * 1e3:.1f}")
 '''
-for v in range(-1, nv):
+for v in vs:
     env = dict(os.environ)
     if v >= 0:
         env["PF_VARIANT"] = str(v)
