@@ -98,6 +98,9 @@ __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t by
       "l"(src), "r"(bytes), "r"(smem_u32(bar))
       : "memory");
 }
+__device__ __forceinline__ void bulk_prefetch_l2(const void* src, uint32_t bytes) {
+  asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(src), "r"(bytes) : "memory");
+}
 __device__ __forceinline__ void mbar_arrive(u64* bar) {
   asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
 }
@@ -736,6 +739,13 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
     if (n >= P.n_local) break;
     if constexpr (C::NSTAGE == 2) {   // prefetch the next sub-filter into the other stage
       if (G.t == 0) issue(st ^ 1, fetch_next());
+    } else {
+      // one stage: the next sub-filter's block is loaded only after this one's
+      // sample loop; pull it from HBM into L2 now, so that load hits L2
+      if (G.t == 0) {
+        const long long nn = gstride + pending;
+        if (nn < P.n_local) bulk_prefetch_l2(P.parts + nn * C::ROW, static_cast<uint32_t>(C::stage_bytes));
+      }
     }
     float* xs = reinterpret_cast<float*>(gs + C::g_stage + st * C::stage_bytes);
     float* ws = xs + D * M;
