@@ -790,16 +790,21 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
       // incoming item j = (neighbour j / t, its j % t-th best): mailbox offset
       // (its log-weight, loaded now, gives the incoming maximum without a
       // dependent shared-memory read after the copy)
-      uint32_t in_max = 0;
-      {
-        uint32_t in_o = 0;
-        if (G.lane < K) {
-          const int qi = static_cast<int>((static_cast<uint32_t>(G.lane) * P.t_inv) >> 16);   // lane / t
-          const int off = static_cast<int>((neighbor_row(P, gsf, qi) * P.tt + (G.lane - qi * P.t)) * E);
-          woff[G.lane] = off;
-          in_o = ord_f32(P.mb_prev[off]);
-        }
-        in_max = __reduce_max_sync(0xFFFFFFFFu, in_o);
+      // All mailbox loads are issued here, before the selection rounds, and
+      // consumed after them: the incoming log-weights (-> incoming maximum)
+      // and this thread's first element of the copy below (one L2 round trip
+      // overlapped with the selection instead of two dependent ones).
+      float in_w = 0.0f, vpre = 0.0f;
+      if (G.lane < K) {
+        const int qi = static_cast<int>((static_cast<uint32_t>(G.lane) * P.t_inv) >> 16);   // lane / t
+        const int off = static_cast<int>((neighbor_row(P, gsf, qi) * P.tt + (G.lane - qi * P.t)) * E);
+        woff[G.lane] = off;
+        in_w = P.mb_prev[off];
+      }
+      __syncwarp();
+      if (G.t < K * E) {
+        const int j = G.t / E;
+        vpre = P.mb_prev[woff[j] + (G.t - j * E)];
       }
       u64 my_cand = ~0ull;
 #pragma unroll 1
@@ -854,10 +859,11 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
         const int s = wlist[j];
         if ((s & (C::T - 1)) == G.t) excl |= 1u << (s / C::T);
       }
+      const uint32_t in_max = __reduce_max_sync(0xFFFFFFFFu, G.lane < K ? ord_f32(in_w) : 0u);
 #pragma unroll 1
       for (int e = G.t; e < K * E; e += C::T) {
         const int j = e / E, c = e - j * E;
-        const float v = P.mb_prev[woff[j] + c];
+        const float v = e == G.t ? vpre : P.mb_prev[woff[j] + c];
         const int slot = wlist[j];
         if (c == 0) ws[slot] = v;
         else if (c >= 2) xs[(c - 2) * M + slot] = v;
