@@ -274,7 +274,7 @@ pf_status pf_get_trace(pf_handle* h, int64_t* src, int32_t* ancestors);
  *   PF_MATH_SINCOS2PI: in uint32 m23[n] -> out float[2n] (sin, cos)  (F3)
  *   PF_MATH_NORMAL_PAIR: in uint32 [x0[n], x1[n]] -> out float[2n] (z0, z1)  (F2)
  *   PF_MATH_PHILOX: in uint32 [c0[n], c1[n], c2[n], c3[n], k0, k1] -> out uint32[4n]  (R12)
- * fn | PF_MATH_X2 (not EXPQ / PHILOX; n even): the same functions evaluated by
+ * fn | PF_MATH_X2 (not PHILOX; n even): the same functions evaluated by
  * the packed f32x2 code path on element pairs (2i, 2i+1), same output layout.
  * No handle; uses the current CUDA device; synchronous. */
 enum { PF_MATH_SIN = 0, PF_MATH_COS = 1, PF_MATH_LOG = 2, PF_MATH_EXPQ = 3, PF_MATH_SQRT = 4,

@@ -56,6 +56,7 @@ __global__ void math_x2_kernel(int fn, const uint32_t* in, uint32_t* out, long l
         out[2 * i + 1] = __float_as_uint(pf::hi2(c)); break;
       case PF_MATH_LOG: s = pf::log_c2(x); out[2 * i] = __float_as_uint(pf::lo2(s));
         out[2 * i + 1] = __float_as_uint(pf::hi2(s)); break;
+      case PF_MATH_EXPQ: pf::expq_c2(x, out[2 * i], out[2 * i + 1]); break;
       case PF_MATH_SQRT: s = pf::sqrt_pos2(x, pf::pk(-__uint_as_float(a), -__uint_as_float(b)));
         out[2 * i] = __float_as_uint(pf::lo2(s)); out[2 * i + 1] = __float_as_uint(pf::hi2(s)); break;
       case PF_MATH_SINCOS2PI: pf::sincos2pi_c2(a, b, s, c);
@@ -91,7 +92,7 @@ pf_status pf_debug_math(int32_t fn_flags, const uint32_t* in, uint32_t* out, int
   const bool x2 = (fn_flags & PF_MATH_X2) != 0;
   const int32_t fn = fn_flags & ~PF_MATH_X2;
   if (!in || !out || n < 0 || fn < PF_MATH_SIN || fn > PF_MATH_PHILOX) return PF_EINVAL;
-  if (x2 && ((n & 1) || fn == PF_MATH_EXPQ || fn == PF_MATH_PHILOX)) return PF_EINVAL;
+  if (x2 && ((n & 1) || fn == PF_MATH_PHILOX)) return PF_EINVAL;
   const long long in_words = fn == PF_MATH_NORMAL_PAIR ? 2 * n : fn == PF_MATH_PHILOX ? 4 * n + 2 : n;
   const long long out_words = (fn == PF_MATH_SINCOS2PI || fn == PF_MATH_NORMAL_PAIR) ? 2 * n
                               : fn == PF_MATH_PHILOX                                  ? 4 * n

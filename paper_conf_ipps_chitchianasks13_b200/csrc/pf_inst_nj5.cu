@@ -22,3 +22,13 @@ const KernelEntry kEntriesNJ5[] = {
 };
 const int kNumEntriesNJ5 = sizeof(kEntriesNJ5) / sizeof(kEntriesNJ5[0]);
 }  // namespace pf
+
+#ifdef PF_TIMELINE
+extern "C" int pf_debug_timeline(unsigned long long* out, long long cap, int reset) {
+  if (reset) {
+    static unsigned long long zero = 0;
+    return cudaMemcpyToSymbol(pf::pf_tl, &zero, sizeof(zero)) == cudaSuccess ? 0 : -3;
+  }
+  return cudaMemcpyFromSymbol(out, pf::pf_tl, sizeof(unsigned long long) * cap) == cudaSuccess ? 0 : -3;
+}
+#endif

@@ -114,6 +114,19 @@ __device__ __forceinline__ void mbar_wait(u64* bar, uint32_t parity) {
       : "memory");
 }
 
+#ifdef PF_TIMELINE
+// dev-only timeline (scripts/timeline.py): one record of 8 u64 per sub-filter
+__device__ unsigned long long pf_tl[1 + 8 * 65536];
+__device__ __forceinline__ unsigned long long tl_now() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+#define TL(v) unsigned long long v = tl_now()
+#else
+#define TL(v)
+#endif
+
 // ------------------------------------------------------- configuration
 // NJ joints (D = NJ + 4), M particles per sub-filter, resampler RES; a group
 // of GW warps owns one sub-filter; S groups per CTA; NSTAGE TMA stages per
@@ -732,9 +745,12 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
   }
   __syncthreads();
 
+  TL(tl_start);
   for (int it = 0;; ++it) {
     const int st = (C::NSTAGE == 2) ? (it & 1) : 0;
+    TL(tl_w0);
     mbar_wait(bars + st, C::NSTAGE == 2 ? (it >> 1) & 1 : it & 1);
+    TL(tl_ready);
     const long long n = next_s[st];
     if (n >= P.n_local) break;
     if constexpr (C::NSTAGE == 2) {   // prefetch the next sub-filter into the other stage
@@ -899,6 +915,7 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
       finish();
       continue;
     }
+    TL(tl_merged);
 
     // ---- a7 normalise + a8 resample (slot order, R11)
     int anc[PP];
@@ -936,8 +953,13 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
           lmax_o = mo;
         }
         const float lmax = unord_f32(lmax_o);
+        if constexpr (PP % 2 == 0) {   // F7 on pairs (packed, bit-identical)
 #pragma unroll
-        for (int j = 0; j < PP; ++j) q[j] = expq_c(lw[j] - lmax);
+          for (int j = 0; j < PP; j += 2) expq_c2(sub2(pk(lw[j], lw[j + 1]), bc(lmax)), q[j], q[j + 1]);
+        } else {
+#pragma unroll
+          for (int j = 0; j < PP; ++j) q[j] = expq_c(lw[j] - lmax);
+        }
         // R21: does this sub-filter resample now?  (uniform in the group)
         if (P.policy == POLICY_ESS) {   // ESS = Q^2 / sum q^2 < tau m, exactly in integers
           u64 s1 = 0, s2 = 0;
@@ -982,6 +1004,7 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
       }
     }
 
+    TL(tl_res);
     if (C::X2 && do_sample) {
       // ---- a9 gather (smem) + a1 RNG + a2 sample + a3 weight + a10 store,
       //      two particles (slots j, j+1 of this thread) at a time with the
@@ -1078,6 +1101,7 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
       }
     }
 
+    TL(tl_smp);
     // the stage buffer is no longer read (new states live in HBM, new
     // log-weights in the scan buffer): start the next sub-filter's load now
     if (C::EARLY && do_sample) release_stage();
@@ -1126,6 +1150,20 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
       }
     }
     finish();
+#ifdef PF_TIMELINE
+    if (G.t == 0) {
+      const unsigned long long tl_end = tl_now();
+      unsigned int smid;
+      asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+      const unsigned long long i = atomicAdd(&pf_tl[0], 1ull);
+      if (i < 65536) {
+        unsigned long long* r = pf_tl + 1 + 8 * i;
+        r[0] = static_cast<unsigned long long>(n) | (static_cast<unsigned long long>(smid) << 32) |
+               (static_cast<unsigned long long>(blockIdx.x * C::S + g) << 40);
+        r[1] = tl_start; r[2] = tl_w0; r[3] = tl_ready; r[4] = tl_merged; r[5] = tl_res; r[6] = tl_smp; r[7] = tl_end;
+      }
+    }
+#endif
   }
 
   // ---- a5: the last CTA to finish copies the winning particle (R6)

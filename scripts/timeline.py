@@ -1,0 +1,54 @@
+"""Dev tool: per-sub-filter timeline of one step-kernel launch (needs a PF_TIMELINE
+build loaded through PF_LIB, see build_variant.py).  usage: timeline.py nj m N res [flush]
+Prints the kernel span, the ramp (first data arrival), mean phase durations per
+sub-filter and the tail (how long the last 10% of groups run alone)."""
+import ctypes as C, os, sys
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import numpy as np, torch
+from paper_conf_ipps_chitchianasks13_b200 import binding, filter as F, workload as W
+
+nj, m, N, res = int(sys.argv[1]), int(sys.argv[2]), int(sys.argv[3]), sys.argv[4]
+flush_l2 = len(sys.argv) <= 5 or sys.argv[5] != "0"
+tr = W.make_trajectory(nj, 20, 0)
+g = F.ParticleFilter(tr["mu0"], tr["sigma0"], F.ArmModel(n_joints=nj), m=m, n_filters=N, resampler=res,
+                     device_inputs=True)
+zs = torch.tensor(tr["Z"][1:], device="cuda"); us = torch.tensor(tr["U"][:-1], device="cuda")
+L = binding.lib()
+fn = L.pf_debug_timeline
+fn.argtypes = [C.c_void_p, C.c_longlong, C.c_int]
+flush = torch.empty(512 << 20, dtype=torch.uint8, device="cuda")
+for k in range(5):
+    g.step(zs[k], us[k])
+torch.cuda.synchronize()
+for rep in range(3):
+    if flush_l2:
+        flush.zero_()
+    torch.cuda.synchronize()
+    fn(None, 0, 1)
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(g.stream); g.step(zs[5 + rep], us[5 + rep]); e1.record(g.stream)
+    torch.cuda.synchronize()
+    buf = np.zeros(1 + 8 * 65536, np.uint64)
+    fn(buf.ctypes.data, buf.size, 0)
+    n = int(buf[0]); r = buf[1:1 + 8 * n].reshape(n, 8).astype(np.int64)
+    t0 = r[:, 1].min()
+    start, w0, ready, merged, resd, smp, end = (r[:, i] - t0 for i in range(1, 8))
+    grp = (r[:, 0] >> 40)
+    span = end.max()
+    print(f"rep {rep}: event {e0.elapsed_time(e1)*1e3:.1f} us, kernel span (first CTA start -> last sub-filter end) {span/1e3:.1f} us, "
+          f"{n} sub-filters, {len(np.unique(grp))} groups")
+    print(f"  CTA start spread {np.ptp(start)/1e3:.2f} us; first data ready {ready.min()/1e3:.2f} us, "
+          f"median first ready {np.median([ready[grp == q].min() for q in np.unique(grp)])/1e3:.2f} us")
+    print(f"  per sub-filter (mean us): wait {np.mean(ready - w0)/1e3:.2f}  exchange {np.mean(merged - ready)/1e3:.2f}  "
+          f"resample {np.mean(resd - merged)/1e3:.2f}  sample {np.mean(smp - resd)/1e3:.2f}  reduce+finish {np.mean(end - smp)/1e3:.2f}"
+          f"  total {np.mean(end - ready)/1e3:.2f}")
+    ends = np.sort([end[grp == q].max() for q in np.unique(grp)])
+    print(f"  group end times (us): p10 {ends[len(ends)//10]/1e3:.1f} p50 {ends[len(ends)//2]/1e3:.1f} "
+          f"p90 {ends[9*len(ends)//10]/1e3:.1f} max {ends[-1]/1e3:.1f}")
+    cnt = np.bincount(np.unique(grp, return_inverse=True)[1])
+    print(f"  sub-filters per group: {np.bincount(cnt)}")
+    # concurrency profile: busy groups in 2-us bins
+    bins = np.arange(0, span + 2000, 2000)
+    busy = [int(np.sum((ready <= b + 1000) & (end > b + 1000))) for b in bins[:-1]]
+    print("  busy sub-filters per 2 us:", busy)
+g.close()

@@ -31,7 +31,9 @@ def test_sqrt_exhaustive_on_box_muller_domain(B):
 @pytest.mark.parametrize("fn", ["sin", "cos"])
 def test_sincos_bit_exact(B, orc, fn, x2):
     rng = np.random.default_rng(1)
-    x = np.concatenate([rng.uniform(-4, 4, 3000), rng.uniform(-60, 60, 3000), [0.0, -0.0, 0.7853981, 1e-30]])
+    # F5 domain |x| < 2^22 pi/2 (the quadrant index fits the 1.5 2^23 rounding add)
+    x = np.concatenate([rng.uniform(-4, 4, 3000), rng.uniform(-60, 60, 3000), rng.uniform(-6.5e6, 6.5e6, 1000),
+                        [0.0, -0.0, 0.7853981, 1e-30, 2.3561945, -2.3561945, 3.926991, -5.497787]])
     x = x.astype(np.float32)
     got = B.pf_debug_math(fn, _f32bits(x), len(x), x2).view(np.float32)
     ref = np.array([orc.s_sin(float(v)) if fn == "sin" else orc.s_cos(float(v)) for v in x], np.float32)
@@ -48,10 +50,12 @@ def test_log_bit_exact(B, orc, x2):
     np.testing.assert_array_equal(got.view(np.uint32), ref.view(np.uint32))
 
 
-def test_expq_bit_exact(B, orc):
+@pytest.mark.parametrize("x2", [False, True], ids=["scalar", "packed"])
+def test_expq_bit_exact(B, orc, x2):
     rng = np.random.default_rng(3)
-    d = np.concatenate([-rng.exponential(3.0, 5000), [0.0, -16.0, -16.0001, -15.25, -1e-8]]).astype(np.float32)
-    got = B.pf_debug_math("expq", _f32bits(d), len(d))
+    d = np.concatenate([-rng.exponential(3.0, 5000), [0.0, -16.0, -16.0001, -15.25, -1e-8, -0.34657359, -1000.0,
+                                                      -0.0]]).astype(np.float32)
+    got = B.pf_debug_math("expq", _f32bits(d), len(d), x2)
     ref = np.array([orc.s_expq(float(v)) for v in d], np.uint32)
     np.testing.assert_array_equal(got, ref)
 
