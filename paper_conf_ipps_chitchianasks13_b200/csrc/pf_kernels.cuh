@@ -401,6 +401,24 @@ __device__ __forceinline__ int upper_bound_u64(const u64* a, int n, u64 x) {
   return lo;
 }
 
+// One level of the RWS binary search over u32 inclusive sums in shared
+// memory: a += INC if sums[a + OFF] <= c (byte addresses).
+template <int OFF, int INC>
+__device__ __forceinline__ void search_step(uint32_t& a, uint32_t c) {
+  asm("{\n\t.reg .pred p;\n\t.reg .u32 v;\n\t"
+      "ld.shared.u32 v, [%0+%2];\n\t"
+      "setp.le.u32 p, v, %1;\n\t"
+      "@p add.u32 %0, %0, %3;\n\t}"
+      : "+r"(a)
+      : "r"(c), "n"(OFF), "n"(INC));
+}
+
+template <int S>
+__device__ __forceinline__ void search_levels(uint32_t& a, uint32_t c) {
+  search_step<4 * (S - 1), 4 * S>(a, c);
+  if constexpr (S > 1) search_levels<S / 2>(a, c);
+}
+
 // ---------------------------------------------------------- resampling
 struct ResampleSmem {
   u64* scan;    // [M] RWS: inclusive sums C (u32 or u64); Vose: D over L, then E over H
@@ -429,11 +447,20 @@ __device__ __forceinline__ void resample_group(const uint32_t (&q)[C::P], const 
 #pragma unroll
     for (int j = 0; j < P; ++j) {
       const X c = static_cast<X>((static_cast<u64>(ua[j]) * Q) >> 32);
-      int pos = 0;
+      if constexpr (C::SCAN32) {
+        // branch-free search on the shared-memory byte address: per level one
+        // LDS at an immediate offset, one compare, one predicated add
+        uint32_t a = smem_u32(Cs);
+        const uint32_t a0 = a;
+        search_levels<M / 2>(a, c);
+        anc[j] = static_cast<int>((a - a0) >> 2);
+      } else {
+        int pos = 0;
 #pragma unroll
-      for (int s = M / 2; s >= 1; s >>= 1)
-        if (Cs[pos + s - 1] <= c) pos += s;
-      anc[j] = pos;
+        for (int s = M / 2; s >= 1; s >>= 1)
+          if (Cs[pos + s - 1] <= c) pos += s;
+        anc[j] = pos;
+      }
     }
   } else {
     // Vose's alias method (PAPER.md:18 §IV, :20–22 §VI-F), table by the
