@@ -163,7 +163,7 @@ struct KCfg {
   static constexpr size_t g_alias = g_prob + (RES == RES_VOSE ? sizeof(u64) * M : 0);
   static constexpr size_t g_lists = g_alias + (RES == RES_VOSE ? sizeof(int) * M : 0);
   static constexpr size_t g_red = g_lists + (RES == RES_VOSE ? sizeof(int) * M : 0);   // u64 [2][32]
-  static constexpr size_t g_cand = g_red + sizeof(u64) * 64;                     // u64 [GW][KMAX+1]
+  static constexpr size_t g_cand = g_red + sizeof(u64) * 64;                     // u64 [GW KMAX + GW]
   static constexpr size_t g_misc = g_cand + sizeof(u64) * GW * (KMAX + 1);       // int [GW][2][KMAX]
   static constexpr size_t g_bar = g_misc + sizeof(int) * GW * 2 * KMAX;          // u64 [2] + next [2]
   static constexpr size_t group_bytes = (g_bar + 32 + 127) / 128 * 128;
@@ -562,22 +562,24 @@ __device__ __forceinline__ void resample_group(const uint32_t (&q)[C::P], const 
 // rows of pf.h pf_shard.  Ring (R3): [g-1, g+1] mod N; 2D torus (R4): [up,
 // down, left, right] with wrap; a shard holds whole grid rows, so left/right
 // are always local and up/down leave the shard only at its first/last row.
-__device__ __forceinline__ long long neighbor_row(const StepParams& P, long long g, int qi) {
-  const long long N = P.n_global;
+__device__ __forceinline__ long long neighbor_row(const StepParams& P, long long g64, int qi) {
+  // 32-bit arithmetic: N m <= 2^32 with m >= 32 keeps every index below 2^27
+  const int N = static_cast<int>(P.n_global), g = static_cast<int>(g64);
+  const int g0 = static_cast<int>(P.g0), nl = static_cast<int>(P.n_local);
   if (P.topo == TOPO_A2A) return P.pool_row;
   if (P.topo == TOPO_RING) {
-    const long long q = qi == 0 ? (g == 0 ? N - 1 : g - 1) : (g == N - 1 ? 0 : g + 1);
-    const long long loc = q - P.g0;
-    if (loc >= 0 && loc < P.n_local) return loc;
-    return qi == 0 ? P.n_local : P.n_local + 1;
+    const int q = qi == 0 ? (g == 0 ? N - 1 : g - 1) : (g == N - 1 ? 0 : g + 1);
+    const int loc = q - g0;
+    if (static_cast<unsigned>(loc) < static_cast<unsigned>(nl)) return loc;
+    return qi == 0 ? nl : nl + 1;
   }
   const int C = static_cast<int>(P.C), R = static_cast<int>(P.R);
-  const int loc = static_cast<int>(g - P.g0);
+  const int loc = g - g0;
   const int lr = loc / C, c = loc - lr * C;
-  const int rows = static_cast<int>(P.n_local / C);
+  const int rows = nl / C;
   switch (qi) {
-    case 0: return lr > 0 ? loc - C : (rows == R ? (R - 1) * C + c : static_cast<int>(P.n_local) + c);
-    case 1: return lr < rows - 1 ? loc + C : (rows == R ? c : static_cast<int>(P.n_local) + C + c);
+    case 0: return lr > 0 ? loc - C : (rows == R ? (R - 1) * C + c : nl + c);
+    case 1: return lr < rows - 1 ? loc + C : (rows == R ? c : nl + C + c);
     case 2: return lr * C + (c == 0 ? C - 1 : c - 1);
     default: return lr * C + (c == C - 1 ? 0 : c + 1);
   }
@@ -715,7 +717,7 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
   G.wig = G.t >> 5;
   G.red = reinterpret_cast<u64*>(gs + C::g_red);
   G.rb = 0;
-  u64* cand = reinterpret_cast<u64*>(gs + C::g_cand);             // [GW][KMAX+1]
+  u64* cand = reinterpret_cast<u64*>(gs + C::g_cand);             // [GW * K] candidates, [GW] maxima at GW * KMAX
   int* wlist = reinterpret_cast<int*>(gs + C::g_misc) + G.wig * 2 * C::KMAX;   // this warp's copy: worst slots
   int* woff = wlist + C::KMAX;                                                  // mailbox offsets of the incoming
 
@@ -865,8 +867,10 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
         lmax_o = wmax;
         if (G.lane < K) wlist[G.lane] = static_cast<int>(0xFFFFFFFFu - static_cast<uint32_t>(my_cand));
       } else {
-        if (G.lane < K) cand[G.wig * (C::KMAX + 1) + G.lane] = my_cand;
-        if (G.lane == 0) cand[G.wig * (C::KMAX + 1) + C::KMAX] = wmax;
+        // flat list: candidate i of the GW * K is cand[i] (warp i / K), the
+        // per-warp maxima after the GW * KMAX candidate slots
+        if (G.lane < K) cand[G.wig * K + G.lane] = my_cand;
+        if (G.lane == 0) cand[GW * C::KMAX + G.wig] = wmax;
         gsync<GW>(g);
         // every warp merges the GW candidate lists (identical result in all warps)
         u64 c[GW];   // candidate i = lane + 32 r of the GW*K list
@@ -874,11 +878,11 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
 #pragma unroll
         for (int r = 0; r < GW; ++r) {
           const int i = G.lane + 32 * r;
-          c[r] = i < ncand ? cand[(i / K) * (C::KMAX + 1) + i % K] : ~0ull;
+          c[r] = i < ncand ? cand[i] : ~0ull;
         }
         uint32_t mo = 0;
 #pragma unroll
-        for (int ww = 0; ww < GW; ++ww) mo = max(mo, static_cast<uint32_t>(cand[ww * (C::KMAX + 1) + C::KMAX]));
+        for (int ww = 0; ww < GW; ++ww) mo = max(mo, static_cast<uint32_t>(cand[GW * C::KMAX + ww]));
         lmax_o = mo;
         u64 mine = ~0ull;
 #pragma unroll 1
