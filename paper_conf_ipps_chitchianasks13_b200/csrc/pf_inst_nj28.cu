@@ -10,8 +10,11 @@ namespace pf {
       PF_ENTRY(NJ, 128, RES, 4, 1, 1, 1, 1), PF_ENTRY(NJ, 256, RES, GW256, 1, 1, 1, MINB256),       \
       PF_ENTRY(NJ, 512, RES, 16, 1, 1, 1, 1), PF_ENTRY(NJ, 1024, RES, 16, 1, 1, 1, 1)
 const KernelEntry kEntriesNJ28[] = {
-    // m = 256 (config C4), measured: RWS two particles per thread (packed f32x2 path), Vose one
-    PF_LARGE_D_ENTRIES(28, 0, 4, 6), PF_LARGE_D_ENTRIES(28, 1, 8, 4),
+    // m = 256 (config C4), measured: two particles per thread (packed f32x2 path with the
+    // chunked joint loop): RWS 6 CTAs of 4 warps per SM, Vose 4 (one particle per thread
+    // was the better Vose mapping before the chunked loop: 1834 -> 1469 us)
+    PF_LARGE_D_ENTRIES(28, 0, 4, 6), PF_LARGE_D_ENTRIES(28, 1, 4, 4),
+    PF_ENTRY(28, 256, 1, 8, 1, 1, 1, 4),
     PF_ENTRY(28, 256, 0, 8, 1, 1, 1, 4),
     PF_ENTRY(28, 256, 0, 8, 1, 1, 1, 3), PF_ENTRY(28, 256, 0, 4, 1, 1, 1, 4), PF_ENTRY(28, 256, 0, 8, 1, 2, 1, 3),
     PF_ENTRY(28, 256, 1, 8, 1, 1, 1, 3), PF_ENTRY(28, 256, 1, 4, 1, 1, 1, 4),

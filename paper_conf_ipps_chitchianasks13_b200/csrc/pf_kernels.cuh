@@ -133,6 +133,9 @@ __device__ __forceinline__ unsigned long long tl_now() {
 // group; the per-particle sample/weight loop over a thread's P slots is
 // unrolled UNR times (P for full unrolling; 1 keeps one copy of the
 // ~10–40 KB per-particle code in the instruction cache).
+#ifndef PF_ROLL_MIN_D
+#define PF_ROLL_MIN_D 16
+#endif
 #ifndef PF_X2_DEFAULT
 #define PF_X2_DEFAULT 1
 #endif
@@ -150,6 +153,10 @@ struct KCfg {
   static constexpr bool SCAN32 = (M <= 512);  // Q <= M 2^22 fits 32 bits
   static constexpr bool STAGED = UNR < P;    // rolled sample loop: per-slot values via smem
   static constexpr bool X2 = X2_ && (P % 2 == 0);   // sample two particles at once (packed f32x2)
+  // large states (the high-DOF arm): the joint chain runs as a loop over
+  // chunks of four joints instead of being unrolled d times, so the
+  // per-particle code fits the instruction cache (ncu: no_instruction stalls)
+  static constexpr bool ROLLED = D > PF_ROLL_MIN_D;
   static_assert(P >= 1 && P * T == M, "M must be a multiple of the group size");
   static_assert(P <= 32, "exclusion masks are 32-bit");
   static_assert(S >= 1 && S <= 15, "named barriers 1..S");
@@ -651,6 +658,102 @@ struct SampleStream2 {
   }
 };
 
+// The same streamed sample + weight as SampleStream / SampleStream2 for large
+// states, with the middle of the joint chain as a runtime loop: pair 0
+// (components 0, 1; block 0 words 2-3 supplied) static, then chunks of four
+// joints 2 + 4i .. 5 + 4i that use exactly Philox block i + 1 (words 4-7 of
+// the chunk), then the remaining components static from pair 1 + 2 NC on.
+// One copy of four joints' code instead of d (instruction cache), identical
+// arithmetic in the same order.
+template <int NJ>
+struct SampleChunked {
+  static constexpr int D = NJ + 4;
+  static constexpr int NC = NJ >= 6 ? (NJ - 2) / 4 : 0;   // chunks of four joints
+  template <typename X>
+  __device__ __forceinline__ static void joint(int c, const ArmConsts& mc, const float* hsu, const float* z, const X& x,
+                                               float xi, ArmAcc& A, float& th) {
+    th = __fmaf_rn(mc.s_th, xi, x(c) + hsu[c]);
+    A.phi = A.phi + th;
+    sincos_c(A.phi, A.s, A.c);
+    A.px = __fmaf_rn(mc.lj, A.c, A.px);
+    A.py = __fmaf_rn(mc.lj, A.s, A.py);
+    const float r = (z[2 + c] - th) * mc.inv_thm;
+    A.acc = __fmaf_rn(r, r, A.acc);   // c >= 2: never the first joint
+  }
+  template <typename X, typename O>
+  __device__ __forceinline__ static void run(const ArmConsts& mc, const float* hsu, const float* z, const X& x,
+                                             NoiseGen& gen, ArmAcc& A, const O& out) {
+    {
+      float z0, z1;
+      gen.template pair<0>(z0, z1);
+      out(0, arm_sample_take<NJ, 0>(mc, hsu, z, x, z0, A));
+      out(1, arm_sample_take<NJ, 1>(mc, hsu, z, x, z1, A));
+    }
+#pragma unroll 1
+    for (int i = 0; i < NC; ++i) {
+      const int c = 2 + 4 * i;
+      const u32x4 b = philox4x32_10_rk(gen.p, gen.k, 0u, static_cast<uint32_t>(i + 1), gen.rk);
+      float n0, n1, n2, n3, th;
+      normal_pair(b.x, b.y, n0, n1);
+      normal_pair(b.z, b.w, n2, n3);
+      joint(c, mc, hsu, z, x, n0, A, th);
+      out(c, th);
+      joint(c + 1, mc, hsu, z, x, n1, A, th);
+      out(c + 1, th);
+      joint(c + 2, mc, hsu, z, x, n2, A, th);
+      out(c + 2, th);
+      joint(c + 3, mc, hsu, z, x, n3, A, th);
+      out(c + 3, th);
+    }
+    SampleStream<NJ, 1 + 2 * NC>::run(mc, hsu, z, x, gen, A, out);
+  }
+};
+
+template <int NJ>
+struct SampleChunked2 {
+  static constexpr int D = NJ + 4;
+  static constexpr int NC = NJ >= 6 ? (NJ - 2) / 4 : 0;
+  template <typename X>
+  __device__ __forceinline__ static void joint(int c, const ArmConsts2& mc, const f2* hsu2, const f2* z2, const X& x,
+                                               f2 xi, ArmAcc2& A, f2& th) {
+    th = fma2(mc.s_th, xi, add2(x(c), hsu2[c]));
+    A.phi = add2(A.phi, th);
+    sincos_c2(A.phi, A.s, A.c);
+    A.px = fma2(mc.lj, A.c, A.px);
+    A.py = fma2(mc.lj, A.s, A.py);
+    const f2 r = mul2(sub2(z2[2 + c], th), mc.inv_thm);
+    A.acc = fma2(r, r, A.acc);   // c >= 2
+  }
+  template <typename X, typename O>
+  __device__ __forceinline__ static void run(const ArmConsts2& mc, const f2* hsu2, const f2* z2, const X& x,
+                                             NoiseGen2& gen, ArmAcc2& A, const O& out) {
+    {
+      f2 z0, z1;
+      gen.template pair<0>(z0, z1);
+      out(0, arm_sample_take2<NJ, 0>(mc, hsu2, z2, x, z0, A));
+      out(1, arm_sample_take2<NJ, 1>(mc, hsu2, z2, x, z1, A));
+    }
+#pragma unroll 1
+    for (int i = 0; i < NC; ++i) {
+      const int c = 2 + 4 * i;
+      const u32x4 ba = philox4x32_10_rk(gen.pa, gen.k, 0u, static_cast<uint32_t>(i + 1), gen.rk);
+      const u32x4 bb = philox4x32_10_rk(gen.pb, gen.k, 0u, static_cast<uint32_t>(i + 1), gen.rk);
+      f2 n0, n1, n2, n3, th;
+      normal_pair2(ba.x, ba.y, bb.x, bb.y, n0, n1);
+      normal_pair2(ba.z, ba.w, bb.z, bb.w, n2, n3);
+      joint(c, mc, hsu2, z2, x, n0, A, th);
+      out(c, th);
+      joint(c + 1, mc, hsu2, z2, x, n1, A, th);
+      out(c + 1, th);
+      joint(c + 2, mc, hsu2, z2, x, n2, A, th);
+      out(c + 2, th);
+      joint(c + 3, mc, hsu2, z2, x, n3, A, th);
+      out(c + 3, th);
+    }
+    SampleStream2<NJ, 1 + 2 * NC>::run(mc, hsu2, z2, x, gen, A, out);
+  }
+};
+
 // All-to-All pool (§VI-E): the best t of `count` mailbox entries
 // (entry e = row e / t, item e % t, E floats [logw, index bits, x]) by the
 // order key of R6, copied to out[0..t) in order.  Whole CTA; t rounds.
@@ -1081,10 +1184,15 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
         NoiseGen2 gen{pbase + static_cast<uint32_t>(sa), pbase + static_cast<uint32_t>(sb), P.k, P.rk,
                       u32x4{0u, 0u, za2, za3}, u32x4{0u, 0u, zb2, zb3}};
         ArmAcc2 A;
-        SampleStream2<NJ, 0>::run(P.mc2, hsu2_s, z2_s, x, gen, A, [outa, outb](int c, f2 v) {
+        auto store2 = [outa, outb](int c, f2 v) {
           outa[c * M] = lo2(v);
           outb[c * M] = hi2(v);
-        });
+        };
+        if constexpr (C::ROLLED) {
+          SampleChunked2<NJ>::run(P.mc2, hsu2_s, z2_s, x, gen, A, store2);
+        } else {
+          SampleStream2<NJ, 0>::run(P.mc2, hsu2_s, z2_s, x, gen, A, store2);
+        }
         f2 l = arm_finish2(P.mc2, z2_s, A);
         if (!resampled) l = add2(pk(c0, c1), l);   // F12
         outa[D * M] = lo2(l);
@@ -1123,6 +1231,7 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
         float* out = gblk + s;
         NoiseGen gen{pbase + static_cast<uint32_t>(s), P.k, P.rk, u32x4{0u, 0u, z2, z3}};
         ArmAcc A;
+        // (one particle per thread: the unrolled chain measured as fast as the chunked one)
         SampleStream<NJ, 0>::run(P.mc, hsu_s, z_s, x, gen, A, [out](int c, float v) { out[c * M] = v; });
         float l = arm_finish(P.mc, z_s, A);
         if (!resampled) l = cr + l;   // F12

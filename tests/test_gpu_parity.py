@@ -130,6 +130,9 @@ def test_full_filter_c1(P, orc, W):
     (5, 128, 64, 1, "torus", "rws"),
     (5, 32, 32, 0, "none", "rws"),
     (28, 64, 8, 1, "ring", "vose"),
+    (28, 256, 8, 1, "ring", "rws"),     # high-DOF arm, packed pairs + chunked joint loop
+    (28, 256, 16, 1, "torus", "vose"),
+    (28, 1024, 2, 3, "ring", "rws"),
     (5, 1024, 4, 4, "torus", "rws"),
     (5, 64, 16, 2, "all2all", "vose"),
     (2, 256, 64, 1, "all2all", "rws"),
