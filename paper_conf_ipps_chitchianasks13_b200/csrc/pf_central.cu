@@ -350,6 +350,11 @@ __global__ void __launch_bounds__(256) cz_step(const CentralParams C) {
       *C.key_next = 0ull;
       *C.counter = 0u;
     }
+    if (C.record_host) {   // completion word polled by pf_estimate (after the record, system scope)
+      __threadfence_system();
+      __syncthreads();
+      if (tid == 0) *reinterpret_cast<volatile uint32_t*>(C.record_host + kRecordSeq) = C.k;
+    }
   }
 }
 

@@ -43,6 +43,11 @@ enum : int { TOPO_NONE = 0, TOPO_RING = 1, TOPO_TORUS = 2, TOPO_A2A = 3 };
 enum : int { RES_RWS = 0, RES_VOSE = 1 };
 enum : int { POLICY_ALWAYS = 0, POLICY_ESS = 1, POLICY_FREQ = 2 };
 
+// mapped host record: [0, 4 + d) the estimate record, [48, 48 + d) the weighted
+// mean, word kRecordSeq the step number of the last record written (pf_estimate
+// polls it instead of synchronizing the stream)
+constexpr int kRecordSeq = 127;
+
 struct StepParams {
   ArmConsts mc;
   ArmConsts2 mc2;          // mc with every field duplicated (packed f32x2 operands)
@@ -1340,6 +1345,11 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
           if (outs[o])
 #pragma unroll
             for (int c = 0; c < 4; ++c) outs[o][c] = r[c];
+      }
+      if (P.record_host) {   // completion word polled by pf_estimate (after the record, system scope)
+        __threadfence_system();
+        __syncthreads();
+        if (tid == 0) *reinterpret_cast<volatile uint32_t*>(P.record_host + kRecordSeq) = P.k;
       }
     }
     if (P.topo == TOPO_A2A && P.t > 0 && mode != MODE_EXCHANGE) {

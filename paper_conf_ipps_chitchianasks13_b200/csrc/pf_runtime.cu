@@ -198,6 +198,8 @@ struct pf_handle {
   bool trace;
   long long* d_src;
   int* d_anc;
+  bool mapped;         // PF_NO_MAPPED unset at init
+  bool last_mapped;    // the last step wrote its record (and step number) into rec_host
   float* rec_host;     // mapped pinned host floats: [0, 4+d) estimate record, [48, 48+d) weighted mean
   float* rec_host_dev; // its device alias
   float* d_reduce_tmp;
@@ -216,6 +218,13 @@ float* inputs(pf_handle* h) { return reinterpret_cast<float*>(h->scratch + kOffI
 
 float* mailbox_parity(pf_handle* h, long long k) {
   return h->mailbox + (k & 1) * h->g.n_ext * h->g.tt * h->g.E;
+}
+
+// Host-input steps of a single-rank filter stream their estimate record into
+// mapped pinned host memory (pf_estimate polls it); device-input steps keep it
+// on the device (record / est_out) and pf_estimate copies it on demand.
+bool streams_record(const pf_handle* h) {
+  return h->mapped && !(h->cfg.flags & PF_DEVICE_INPUTS) && h->cfg.world == 1;
 }
 
 pf::StepParams base_params(pf_handle* h, long long k, int mode) {
@@ -239,7 +248,7 @@ pf::StepParams base_params(pf_handle* h, long long k, int mode) {
   p.counter = reinterpret_cast<unsigned int*>(h->scratch + kOffCounter);
   p.work = reinterpret_cast<unsigned int*>(h->scratch + kOffWork);
   p.record = record(h);
-  p.record_host = std::getenv("PF_NO_MAPPED") ? nullptr : h->rec_host_dev;
+  p.record_host = streams_record(h) ? h->rec_host_dev : nullptr;
   p.est_out = nullptr;
   p.dbg_src = nullptr;
   p.dbg_anc = nullptr;
@@ -321,7 +330,7 @@ pf::CentralParams central_params(pf_handle* h, long long k) {
   c.counter = reinterpret_cast<unsigned int*>(h->scratch + kOffCounter);
   c.record_prev = record(h);
   c.record = record(h);
-  c.record_host = std::getenv("PF_NO_MAPPED") ? nullptr : h->rec_host_dev;
+  c.record_host = streams_record(h) ? h->rec_host_dev : nullptr;
   const uint32_t key0 = static_cast<uint32_t>(h->cfg.seed), key1 = static_cast<uint32_t>(h->cfg.seed >> 32);
   for (int r = 0; r < 10; ++r) {
     c.rk[2 * r] = key0 + static_cast<uint32_t>(r) * 0x9E3779B9u;
@@ -495,6 +504,11 @@ pf_status pf_init(const pf_config* cfg, const pf_model_params* model, const pf_b
   if (e == cudaSuccess)
     e = cudaHostAlloc(reinterpret_cast<void**>(&h->rec_host), sizeof(float) * 128, cudaHostAllocMapped);
   if (e == cudaSuccess) e = cudaHostGetDevicePointer(reinterpret_cast<void**>(&h->rec_host_dev), h->rec_host, 0);
+  if (e == cudaSuccess) {
+    h->mapped = std::getenv("PF_NO_MAPPED") == nullptr;
+    h->last_mapped = false;
+    reinterpret_cast<volatile uint32_t*>(h->rec_host)[pf::kRecordSeq] = 0xFFFFFFFFu;
+  }
   if (e != cudaSuccess) {
     pf_destroy(h);
     return PF_ECUDA;
@@ -566,7 +580,10 @@ pf_status pf_step(pf_handle* h, const float* z_k, const float* u_km1) {
       host_inputs(h, c, z_k, u_km1);
     }
     const pf_status s = launch_central(h, c);
-    if (s == PF_OK) h->step = k;
+    if (s == PF_OK) {
+      h->step = k;
+      h->last_mapped = c.record_host != nullptr;
+    }
     return s;
   }
   pf::StepParams p = base_params(h, k, pf::MODE_STEP);
@@ -581,7 +598,10 @@ pf_status pf_step(pf_handle* h, const float* z_k, const float* u_km1) {
     p.dbg_anc = h->d_anc;
   }
   const pf_status s = launch(h, p);
-  if (s == PF_OK) h->step = k;
+  if (s == PF_OK) {
+    h->step = k;
+    h->last_mapped = p.record_host != nullptr;
+  }
   return s;
 }
 
@@ -590,6 +610,7 @@ pf_status pf_step_batch(pf_handle* h, int32_t T, const float* zs, const float* u
   if (h->err != PF_OK) return h->err;
   if (h->cfg.world != 1) return PF_ESTATE;
   const int nj = h->g.nj;
+  h->last_mapped = false;
   for (int32_t s = 0; s < T; ++s) {
     const long long k = h->step + 1;
     if (h->g.central) {
@@ -597,6 +618,7 @@ pf_status pf_step_batch(pf_handle* h, int32_t T, const float* zs, const float* u
       c.z = zs + static_cast<long long>(s) * (nj + 2);
       c.u = us + static_cast<long long>(s) * nj;
       c.est_out = est ? est + static_cast<long long>(s) * (4 + h->g.d) : nullptr;
+      c.record_host = nullptr;   // device-resident pipeline: records stay on the device
       const pf_status st = launch_central(h, c);
       if (st != PF_OK) return st;
       h->step = k;
@@ -606,6 +628,7 @@ pf_status pf_step_batch(pf_handle* h, int32_t T, const float* zs, const float* u
     p.z = zs + static_cast<long long>(s) * (nj + 2);
     p.u = us + static_cast<long long>(s) * nj;
     p.est_out = est ? est + static_cast<long long>(s) * (4 + h->g.d) : nullptr;
+    p.record_host = nullptr;   // device-resident pipeline: records stay on the device
     if (h->trace) {
       p.dbg_src = h->d_src;
       p.dbg_anc = h->d_anc;
@@ -621,10 +644,30 @@ pf_status pf_estimate(pf_handle* h, float* x_hat, float* logw, int64_t* idx) {
   if (!h || !x_hat) return PF_EINVAL;
   if (h->err != PF_OK) return h->err;
   if (h->step < 1) return PF_ESTATE;
-  // the kernels wrote the record into mapped pinned host memory: a stream
-  // synchronization is the whole device -> host transfer
-  cudaError_t e = cudaStreamSynchronize(h->stream);
-  if (e != cudaSuccess) return sticky(h, e);
+  // Host-input steps (the streaming, real-time use): the kernel wrote the
+  // record into mapped pinned host memory followed by the step number (system-
+  // scope fence in between), so waiting is polling that word — no stream
+  // synchronization on the critical path; a stream that completes without
+  // it (or any error) ends the poll.  Otherwise (device inputs, several
+  // ranks) the record is copied from the device after a stream synchronization.
+  cudaError_t e = cudaSuccess;
+  if (h->last_mapped) {
+    const uint32_t want = static_cast<uint32_t>(h->step);
+    volatile const uint32_t* seq = reinterpret_cast<volatile const uint32_t*>(h->rec_host + pf::kRecordSeq);
+    for (unsigned it = 1; *seq != want; ++it) {
+      if ((it & 1023u) == 0u) {
+        e = cudaStreamQuery(h->stream);
+        if (e != cudaErrorNotReady) break;
+      }
+    }
+    if (e == cudaSuccess || e == cudaErrorNotReady) e = cudaStreamQuery(h->stream);
+    if (e == cudaErrorNotReady) e = cudaSuccess;   // the record is complete; the kernel is retiring
+    if (e != cudaSuccess) return sticky(h, e);
+  } else {
+    e = cudaMemcpyAsync(h->rec_host, record(h), sizeof(float) * (4 + h->g.d), cudaMemcpyDeviceToHost, h->stream);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(h->stream);
+    if (e != cudaSuccess) return sticky(h, e);
+  }
   float rec[4 + 32 + 4];
   std::memcpy(rec, const_cast<const float*>(h->rec_host), sizeof(float) * (4 + h->g.d));
   uint32_t lo;
@@ -765,6 +808,7 @@ pf_status pf_set_particles(pf_handle* h, const float* state_host, const float* l
   pf_status s = publish(h, step);
   if (s != PF_OK) return s;
   h->step = step;
+  h->last_mapped = false;
   return sticky(h, cudaStreamSynchronize(h->stream));
 }
 
@@ -791,6 +835,7 @@ pf_status pf_debug_sample_weight(pf_handle* h, const float* state_in, const floa
   }
   if (s != PF_OK) return s;
   h->step = k;
+  h->last_mapped = false;
   e = cudaStreamSynchronize(h->stream);
   if (e == cudaSuccess)
     e = rows_to_host(h, set_of_step(h, k), state_out, 0, h->g.d);
@@ -852,6 +897,7 @@ pf_status pf_debug_exchange(pf_handle* h, const float* logw, int64_t* src) {
   st = launch(h, p);
   if (st != PF_OK) return st;
   h->step = s;
+  h->last_mapped = false;
   e = cudaStreamSynchronize(h->stream);
   if (e == cudaSuccess) e = cudaMemcpy(src, dsrc.p, sizeof(long long) * M, cudaMemcpyDeviceToHost);
   return sticky(h, e);
