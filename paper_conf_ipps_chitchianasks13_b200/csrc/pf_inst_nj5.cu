@@ -27,8 +27,11 @@ const int kNumEntriesNJ5 = sizeof(kEntriesNJ5) / sizeof(kEntriesNJ5[0]);
 extern "C" int pf_debug_timeline(unsigned long long* out, long long cap, int reset) {
   if (reset) {
     static unsigned long long zero = 0;
+    static unsigned long long init2[4] = {~0ull, 0ull, 0ull, 0ull};
+    if (cudaMemcpyToSymbol(pf::pf_tl2, init2, sizeof(init2)) != cudaSuccess) return -3;
     return cudaMemcpyToSymbol(pf::pf_tl, &zero, sizeof(zero)) == cudaSuccess ? 0 : -3;
   }
+  if (cap < 0) return cudaMemcpyFromSymbol(out, pf::pf_tl2, sizeof(unsigned long long) * 4) == cudaSuccess ? 0 : -3;
   return cudaMemcpyFromSymbol(out, pf::pf_tl, sizeof(unsigned long long) * cap) == cudaSuccess ? 0 : -3;
 }
 #endif

@@ -122,6 +122,7 @@ __device__ __forceinline__ void mbar_wait(u64* bar, uint32_t parity) {
 #ifdef PF_TIMELINE
 // dev-only timeline (scripts/timeline.py): one record of 8 u64 per sub-filter
 __device__ unsigned long long pf_tl[1 + 8 * 65536];
+__device__ unsigned long long pf_tl2[4];   // min CTA entry, last-CTA epilogue start, its end
 __device__ __forceinline__ unsigned long long tl_now() {
   unsigned long long t;
   asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
@@ -801,6 +802,9 @@ __device__ void pool_top_t(const StepParams& P, const float* mb, long long count
 // ------------------------------------------------------------ the kernel
 template <class C>
 __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __grid_constant__ StepParams P) {
+#ifdef PF_TIMELINE
+  if (threadIdx.x == 0) atomicMin(&pf_tl2[0], tl_now());
+#endif
   constexpr int NJ = C::NJ, M = C::M, D = C::D, E = C::E, GW = C::GW, PP = C::P;
   extern __shared__ __align__(128) unsigned char smem[];
   float* z_s = reinterpret_cast<float*>(smem + C::c_zin);
@@ -1312,6 +1316,9 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
   }
 
   // ---- a5: the last CTA to finish copies the winning particle (R6)
+#ifdef PF_TIMELINE
+  const unsigned long long tl_epi = tl_now();
+#endif
   __shared__ unsigned int s_last;
   __syncthreads();
   if (threadIdx.x == 0) {
@@ -1371,6 +1378,10 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
     if (tid == 0) {
       *P.key_next = 0ull;
       *P.counter = 0u;
+#ifdef PF_TIMELINE
+      pf_tl2[1] = tl_epi;
+      pf_tl2[2] = tl_now();
+#endif
       *P.work = 0u;
     }
   }

@@ -103,6 +103,15 @@ class ParticleFilter:
         self.central = n_filters == 1 and m > 1024
         self._k = 0
         self._xhat = np.zeros(self.d, np.float32)
+        # per-step host path (e2e): persistent input / output buffers with
+        # their pointers taken once (numpy pointer extraction costs ~1 us)
+        self._device_inputs = bool(self.cfg.flags & B.PF_DEVICE_INPUTS)
+        self._zin = np.zeros(self.nj + 2, np.float32)
+        self._uin = np.zeros(self.nj, np.float32)
+        self._zin_p, self._uin_p, self._xhat_p = self._zin.ctypes.data, self._uin.ctypes.data, self._xhat.ctypes.data
+        self._step_fn, self._est_fn = B.lib().pf_step, B.lib().pf_estimate
+        self._lw, self._idx = B.C.c_float(), B.C.c_int64()
+        self._lw_ref, self._idx_ref = B.C.byref(self._lw), B.C.byref(self._idx)
 
     # -- views of the caller-owned buffers (torch, device) -------------------
     @property
@@ -128,10 +137,14 @@ class ParticleFilter:
     # -- the path -----------------------------------------------------------
     def step(self, z, u) -> None:
         """One time step (host numpy z/u, or device tensors with device_inputs)."""
-        if self.cfg.flags & B.PF_DEVICE_INPUTS:
-            B.pf_step(self.h, z.data_ptr(), u.data_ptr())
-        else:
-            B.pf_step(self.h, _f32(z), _f32(u))
+        if self._device_inputs:
+            st = self._step_fn(self.h, z.data_ptr(), u.data_ptr())
+        else:   # copied into the launch by pf_step (R-contract: host inputs travel with the kernel)
+            np.copyto(self._zin, z, casting="same_kind")
+            np.copyto(self._uin, u, casting="same_kind")
+            st = self._step_fn(self.h, self._zin_p, self._uin_p)
+        if st != B.PF_OK:
+            B.check(st, "pf_step")
         self._k += 1
 
     def step_batch(self, zs: torch.Tensor, us: torch.Tensor, est: torch.Tensor | None = None) -> None:
@@ -142,8 +155,10 @@ class ParticleFilter:
 
     def estimate(self):
         """(x_hat [d], logw, global index) of the particle with the highest weight."""
-        lw, idx = B.pf_estimate(self.h, self._xhat)
-        return self._xhat.copy(), lw, idx
+        st = self._est_fn(self.h, self._xhat_p, self._lw_ref, self._idx_ref)
+        if st != B.PF_OK:
+            B.check(st, "pf_estimate")
+        return self._xhat.copy(), self._lw.value, self._idx.value
 
     def estimate_mean(self) -> np.ndarray:
         """Weighted-average estimate x [d] of the last step's set (R22; §VI-D)."""

@@ -30,7 +30,12 @@ for rep in range(3):
     torch.cuda.synchronize()
     buf = np.zeros(1 + 8 * 65536, np.uint64)
     fn(buf.ctypes.data, buf.size, 0)
+    t2 = np.zeros(4, np.uint64)
+    fn(t2.ctypes.data, -1, 0)
     n = int(buf[0]); r = buf[1:1 + 8 * n].reshape(n, 8).astype(np.int64)
+    tmin = int(r[:, 1].min())
+    print(f"  first CTA entry -> first group start {(tmin - int(t2[0]))/1e3:.2f} us; last group end -> "
+          f"epilogue (last CTA) start {(int(t2[1]) - int(r[:, 7].max()))/1e3:.2f} us; epilogue {(int(t2[2]) - int(t2[1]))/1e3:.2f} us")
     t0 = r[:, 1].min()
     start, w0, ready, merged, resd, smp, end = (r[:, i] - t0 for i in range(1, 8))
     grp = (r[:, 0] >> 40)
