@@ -68,6 +68,8 @@ struct StepParams {
   long long n_local, g0, n_global, R, C;
   long long pool_row;      // All-to-All: the row every sub-filter reads (global best t)
   long long pool_local_row;  // All-to-All: where the last CTA writes this shard's best t
+  u64* pool_cta;             // All-to-All, t >= 2: [gridDim][tt] x {order key, mailbox entry} of each
+                             // CTA's best t (the last CTA merges these instead of the whole mailbox)
   int t, tt, topo, deg;
   uint32_t t_inv;          // ceil(2^16 / t): lane / t = (lane * t_inv) >> 16 for lane < 2^16 / t
   uint32_t k;
@@ -760,6 +762,74 @@ struct SampleChunked2 {
   }
 };
 
+// Best t of the union of two descending lists held by lanes 0..t-1 (run list
+// r, new list nb; keys unique or 0 = empty) into r, by t rounds of warp max.
+__device__ __forceinline__ void top_t_merge(u64& rk, u64& rl, u64 nk, u64 nl, int t, int lane) {
+  u64 a = lane < t ? rk : 0ull, b = lane < t ? nk : 0ull;
+  u64 ok = 0ull, ol = 0ull;
+  for (int r = 0; r < t; ++r) {
+    const u64 c = a > b ? a : b;
+    const u64 w = warp_max_u64(c);
+    const bool own = w != 0ull && c == w;
+    const int owner = __ffs(__ballot_sync(0xFFFFFFFFu, own)) - 1;
+    const u64 wl = __shfl_sync(0xFFFFFFFFu, a == w ? rl : nl, owner < 0 ? 0 : owner);
+    if (own) {
+      if (a == w) a = 0ull;
+      else b = 0ull;
+    }
+    if (lane == r) {
+      ok = w;
+      ol = owner < 0 ? 0ull : wl;
+    }
+  }
+  rk = ok;
+  rl = ol;
+}
+
+// All-to-All pool from the per-CTA best t (pool_cta): the best t of the
+// gridDim * t candidates, entries copied from the mailbox.  Whole CTA.
+template <int E>
+__device__ void pool_top_t_cta(const StepParams& P, float* out) {
+  __shared__ u64 red_k[33], red_l[33];
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5, nw = (blockDim.x + 31) >> 5;
+  const long long count = static_cast<long long>(gridDim.x) * P.tt;
+  u64 prev = ~0ull;
+  for (int jb = 0; jb < P.t; ++jb) {
+    u64 best = 0ull, bl = 0ull;
+    for (long long i = tid; i < count; i += blockDim.x) {
+      const u64 key = __ldcg(P.pool_cta + 2 * i);
+      if (key < prev && key > best) {
+        best = key;
+        bl = __ldcg(P.pool_cta + 2 * i + 1);
+      }
+    }
+    const u64 wbest = warp_max_u64(best);
+    if (best == wbest && wbest != 0ull) {   // unique owner in the warp
+      red_k[warp] = wbest;
+      red_l[warp] = bl;
+    } else if (lane == 0 && wbest == 0ull) {
+      red_k[warp] = 0ull;
+    }
+    __syncthreads();
+    if (warp == 0) {
+      const u64 k = lane < nw ? red_k[lane] : 0ull;
+      const u64 v = warp_max_u64(k);
+      if (v != 0ull && k == v) {
+        red_k[32] = v;
+        red_l[32] = red_l[lane];
+      }
+      if (lane == 0 && v == 0ull) red_k[32] = 0ull;
+    }
+    __syncthreads();
+    const u64 g = red_k[32];
+    const float* en = P.mb_cur + static_cast<long long>(red_l[32]) * E;
+    if (g != 0ull)
+      for (int c = tid; c < E; c += blockDim.x) out[jb * E + c] = __ldcg(en + c);
+    prev = g;
+    __syncthreads();
+  }
+}
+
 // All-to-All pool (§VI-E): the best t of `count` mailbox entries
 // (entry e = row e / t, item e % t, E floats [logw, index bits, x]) by the
 // order key of R6, copied to out[0..t) in order.  Whole CTA; t rounds.
@@ -833,6 +903,9 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
   int* wlist = reinterpret_cast<int*>(gs + C::g_misc) + G.wig * 2 * C::KMAX;   // this warp's copy: worst slots
   int* woff = wlist + C::KMAX;                                                  // mailbox offsets of the incoming
 
+  // All-to-All t >= 2: this group's running best t over its sub-filters
+  // (lane j < t of warp 0 holds the j-th: order key, mailbox entry index)
+  u64 gtop_k = 0ull, gtop_l = 0ull;
   const int mode = P.mode;
   const bool do_merge = (mode == MODE_EXCHANGE) || (mode == MODE_STEP && !P.first);
   const bool do_resample = (mode == MODE_STEP && !P.first);
@@ -1263,6 +1336,7 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
         lnew[j] = do_sample ? reinterpret_cast<const float*>(bzw_s)[2 * C::slot(G.t, j)] : lw[j];
       uint32_t done = 0;
       const int nbest = P.t > 0 ? P.t : 1;
+      u64 nb_k = 0ull, nb_l = 0ull;
 #pragma unroll 1
       for (int jb = 0; jb < nbest; ++jb) {
         u64 mk = 0ull;
@@ -1272,6 +1346,10 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
           mk = key > mk ? key : mk;
         }
         const u64 best = gmax_u64<GW>(mk, G);
+        if (G.lane == jb) {   // this sub-filter's jb-th best (uniform in the group)
+          nb_k = best;
+          nb_l = static_cast<u64>(n * P.tt + jb);
+        }
         const int bslot = static_cast<int>(0xFFFFFFFFu - static_cast<uint32_t>(best) - pbase);
 #pragma unroll
         for (int j = 0; j < PP; ++j) {
@@ -1297,6 +1375,7 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
           }
         }
       }
+      if (P.pool_cta && G.wig == 0) top_t_merge(gtop_k, gtop_l, nb_k, nb_l, P.t, G.lane);
     }
     finish();
 #ifdef PF_TIMELINE
@@ -1313,6 +1392,50 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
       }
     }
 #endif
+  }
+
+  // ---- All-to-All t >= 2: the CTA's best t of its groups' lists -> pool_cta
+  //      (the stage buffers are free: no load is in flight after the loop)
+  if (P.pool_cta) {
+    u64* lists = reinterpret_cast<u64*>(gs + C::g_stage);   // this group's [t] keys, then [t] entries
+    if (G.wig == 0 && G.lane < P.t) {
+      lists[G.lane] = gtop_k;
+      lists[P.t + G.lane] = gtop_l;
+    }
+    __syncthreads();
+    if (threadIdx.x < 32) {
+      // candidate i = group i / t, item i % t; S * t <= 15 * 32
+      u64 ck = 0ull, cl = 0ull;
+      for (int r = 0; r < P.t; ++r) {
+        u64 mine = 0ull;
+        int mi = -1;
+        for (int i = threadIdx.x; i < C::S * P.t; i += 32) {
+          const int gg = i / P.t, jj = i - gg * P.t;
+          const u64 kk = reinterpret_cast<u64*>(smem + C::c_groups + gg * C::group_bytes + C::g_stage)[jj];
+          if (kk > mine) {
+            mine = kk;
+            mi = i;
+          }
+        }
+        const u64 w = warp_max_u64(mine);
+        if (w != 0ull && mine == w) {   // unique owner (keys carry the particle index)
+          const int gg = mi / P.t, jj = mi - gg * P.t;
+          u64* gl = reinterpret_cast<u64*>(smem + C::c_groups + gg * C::group_bytes + C::g_stage);
+          ck = w;
+          cl = gl[P.t + jj];
+          gl[jj] = 0ull;
+        }
+        __syncwarp();
+        const int owner = __ffs(__ballot_sync(0xFFFFFFFFu, w != 0ull && mine == w)) - 1;
+        const u64 wl = owner >= 0 ? __shfl_sync(0xFFFFFFFFu, cl, owner) : 0ull;
+        if (threadIdx.x == 0) {
+          P.pool_cta[(static_cast<long long>(blockIdx.x) * P.tt + r) * 2] = w;
+          P.pool_cta[(static_cast<long long>(blockIdx.x) * P.tt + r) * 2 + 1] = wl;
+        }
+        __syncwarp();
+      }
+      (void)ck;
+    }
   }
 
   // ---- a5: the last CTA to finish copies the winning particle (R6)
@@ -1371,6 +1494,8 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
           pool[0] = unord_f32(static_cast<uint32_t>(key >> 32));
           pool[1] = __uint_as_float(gidx);
         }
+      } else if (P.pool_cta) {
+        pool_top_t_cta<E>(P, pool);
       } else {
         pool_top_t<E>(P, P.mb_cur, P.n_local * P.t, pool);
       }

@@ -220,6 +220,13 @@ float* mailbox_parity(pf_handle* h, long long k) {
   return h->mailbox + (k & 1) * h->g.n_ext * h->g.tt * h->g.E;
 }
 
+// All-to-All with t >= 2: per-CTA best-t candidates after the mailbox parities
+// ({order key, entry} u64 pairs for up to kPoolCtas CTAs of the step kernel).
+constexpr long long kPoolCtas = 8192;
+size_t pool_cta_bytes(const pf_config* cfg, const Geometry& g) {
+  return (!g.central && cfg->topo == PF_TOPO_ALL2ALL && cfg->t >= 2) ? sizeof(u64) * 2 * kPoolCtas * g.tt : 0;
+}
+
 // Host-input steps of a single-rank filter stream their estimate record into
 // mapped pinned host memory (pf_estimate polls it); device-input steps keep it
 // on the device (record / est_out) and pf_estimate copies it on demand.
@@ -259,6 +266,9 @@ pf::StepParams base_params(pf_handle* h, long long k, int mode) {
   p.C = h->g.C;
   p.pool_row = h->g.n_local + (h->cfg.world > 1 ? h->cfg.world : 0);
   p.pool_local_row = h->g.n_local + (h->cfg.world > 1 ? h->cfg.rank : 0);
+  p.pool_cta = pool_cta_bytes(&h->cfg, h->g)
+                   ? reinterpret_cast<u64*>(h->mailbox + 2 * h->g.n_ext * h->g.tt * h->g.E)
+                   : nullptr;
   p.t = h->cfg.t;
   p.t_inv = h->cfg.t > 0 ? (65536u + static_cast<uint32_t>(h->cfg.t) - 1u) / static_cast<uint32_t>(h->cfg.t) : 0u;
   p.tt = h->g.tt;
@@ -457,7 +467,7 @@ pf_status pf_query_sizes(const pf_config* cfg, const pf_model_params* model, pf_
   const pf_status s = validate(cfg, model, &g);
   if (s != PF_OK || !out) return s != PF_OK ? s : PF_EINVAL;
   out->state = g.central ? central_bytes(g) : sizeof(float) * g.ROW * g.n_local;
-  out->mailbox = sizeof(float) * 2 * g.n_ext * g.tt * g.E;
+  out->mailbox = sizeof(float) * 2 * g.n_ext * g.tt * g.E + pool_cta_bytes(cfg, g);
   out->scratch = kScratchBytes;
   return PF_OK;
 }
@@ -539,6 +549,7 @@ pf_status pf_init(const pf_config* cfg, const pf_model_params* model, const pf_b
     const long long ctas_needed = (g.n_local + h->ke->s - 1) / h->ke->s;
     const long long grid = static_cast<long long>(bps) * sms;
     h->grid = static_cast<int>(grid < ctas_needed ? grid : ctas_needed);
+    if (pool_cta_bytes(cfg, g) && h->grid > kPoolCtas) h->grid = static_cast<int>(kPoolCtas);
   }
   // scratch: zero keys / counter; prior parameters
   float prior[128];

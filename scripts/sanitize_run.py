@@ -6,7 +6,7 @@ import numpy as np
 from paper_conf_ipps_chitchianasks13_b200 import filter as F, workload as W
 
 cases = [(2, 64, 16, 1, "ring", "rws"), (5, 256, 8, 2, "torus", "vose"), (5, 32, 16, 1, "all2all", "rws"),
-         (5, 256, 64, 1, "ring", "rws"), (28, 256, 4, 1, "ring", "vose"), (5, 1024, 4, 3, "torus", "rws"),
+         (5, 256, 64, 1, "ring", "rws"), (28, 256, 4, 1, "ring", "vose"), (28, 256, 4, 1, "ring", "rws"), (5, 1024, 4, 3, "torus", "rws"),
          (5, 128, 16, 2, "all2all", "vose")]
 for nj, m, N, t, topo, res in cases:
     tr = W.make_trajectory(nj, 6, 1)
