@@ -68,8 +68,8 @@ struct StepParams {
   long long n_local, g0, n_global, R, C;
   long long pool_row;      // All-to-All: the row every sub-filter reads (global best t)
   long long pool_local_row;  // All-to-All: where the last CTA writes this shard's best t
-  u64* pool_cta;             // All-to-All, t >= 2: [gridDim][tt] x {order key, mailbox entry} of each
-                             // CTA's best t (the last CTA merges these instead of the whole mailbox)
+  u64* pool_cta;             // All-to-All, t >= 2: [groups][tt] x {order key, mailbox entry}: each
+                             // group's best t (the last CTA merges these instead of the whole mailbox)
   int t, tt, topo, deg;
   uint32_t t_inv;          // ceil(2^16 / t): lane / t = (lane * t_inv) >> 16 for lane < 2^16 / t
   uint32_t k;
@@ -541,13 +541,30 @@ __device__ __forceinline__ void resample_group(const uint32_t (&q)[C::P], const 
       int ls;
       cls(j, small, a, Dinc, Einc, ls);
       const int s = C::slot(G.t, j);
+      // one branch-free search per slot, the same for small and large slots
+      // (no divergence between them): small -> first E over H that is >=
+      // D_{i-1}; large with E < D_last -> first D over L that is > E, i.e.
+      // >= E + 1 (integers).  log2(M) predicated halving steps.
+      const bool srch = small || Einc < Dtot;
+      const u64 key = small ? Dinc - (Qg - a) : Einc + 1;
+      int base = small ? nL : 0;
+      int len = !srch ? 1 : (small ? M - nL : nL);
+#pragma unroll
+      for (int it = 1; it < M; it <<= 1) {
+        if (len > 1) {
+          const int half = len >> 1;
+          if (S.scan[base + half] < key) base += half;
+          len -= half;
+        }
+      }
+      const int pos = base + (srch && S.scan[base] < key ? 1 : 0);   // absolute index in scan / lists
       u64 pr;
       int al;
       if (small) {
         pr = a;
-        al = S.lists[nL + lower_bound_u64(S.scan + nL, M - nL, Dinc - (Qg - a))];
-      } else if (Einc < Dtot) {
-        pr = Qg + Einc - S.scan[upper_bound_u64(S.scan, nL, Einc)];
+        al = S.lists[pos];
+      } else if (srch) {
+        pr = Qg + Einc - S.scan[pos];
         al = S.lists[nL + (s - ls) + 1];
       } else {
         pr = Qg;
@@ -786,13 +803,15 @@ __device__ __forceinline__ void top_t_merge(u64& rk, u64& rl, u64 nk, u64 nl, in
   rl = ol;
 }
 
-// All-to-All pool from the per-CTA best t (pool_cta): the best t of the
-// gridDim * t candidates, entries copied from the mailbox.  Whole CTA.
+// All-to-All pool from the per-group best t (pool_cta rows of the groups
+// that processed a sub-filter: static first index gid0 < n_local): the best t
+// of those candidates, entries copied from the mailbox.  Whole CTA.
 template <int E>
-__device__ void pool_top_t_cta(const StepParams& P, float* out) {
-  __shared__ u64 red_k[33], red_l[33];
+__device__ void pool_top_t_cta(const StepParams& P, float* out, u64* red, long long groups) {   // red: 66 u64
+  u64* red_k = red;
+  u64* red_l = red + 33;
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5, nw = (blockDim.x + 31) >> 5;
-  const long long count = static_cast<long long>(gridDim.x) * P.tt;
+  const long long count = (groups < P.n_local ? groups : P.n_local) * P.tt;
   u64 prev = ~0ull;
   for (int jb = 0; jb < P.t; ++jb) {
     u64 best = 0ull, bl = 0ull;
@@ -834,8 +853,7 @@ __device__ void pool_top_t_cta(const StepParams& P, float* out) {
 // (entry e = row e / t, item e % t, E floats [logw, index bits, x]) by the
 // order key of R6, copied to out[0..t) in order.  Whole CTA; t rounds.
 template <int E>
-__device__ void pool_top_t(const StepParams& P, const float* mb, long long count, float* out) {
-  __shared__ u64 pool_red[33];
+__device__ void pool_top_t(const StepParams& P, const float* mb, long long count, float* out, u64* pool_red) {
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5, nw = (blockDim.x + 31) >> 5;
   u64 prev = ~0ull;
   for (int jb = 0; jb < P.t; ++jb) {
@@ -903,9 +921,6 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
   int* wlist = reinterpret_cast<int*>(gs + C::g_misc) + G.wig * 2 * C::KMAX;   // this warp's copy: worst slots
   int* woff = wlist + C::KMAX;                                                  // mailbox offsets of the incoming
 
-  // All-to-All t >= 2: this group's running best t over its sub-filters
-  // (lane j < t of warp 0 holds the j-th: order key, mailbox entry index)
-  u64 gtop_k = 0ull, gtop_l = 0ull;
   const int mode = P.mode;
   const bool do_merge = (mode == MODE_EXCHANGE) || (mode == MODE_STEP && !P.first);
   const bool do_resample = (mode == MODE_STEP && !P.first);
@@ -1346,7 +1361,7 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
           mk = key > mk ? key : mk;
         }
         const u64 best = gmax_u64<GW>(mk, G);
-        if (G.lane == jb) {   // this sub-filter's jb-th best (uniform in the group)
+        if (P.pool_cta && G.lane == jb) {   // All-to-All t >= 2: this sub-filter's jb-th best
           nb_k = best;
           nb_l = static_cast<u64>(n * P.tt + jb);
         }
@@ -1375,7 +1390,22 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
           }
         }
       }
-      if (P.pool_cta && G.wig == 0) top_t_merge(gtop_k, gtop_l, nb_k, nb_l, P.t, G.lane);
+      if (P.pool_cta && G.wig == 0) {
+        // All-to-All t >= 2: merge this sub-filter's best t into the group's
+        // running best t (global row of the group, lanes < t; empty before
+        // the group's first sub-filter)
+        u64* row = P.pool_cta + (gid0 * P.tt + G.lane) * 2;
+        u64 rk = 0ull, rl = 0ull;
+        if (it > 0 && G.lane < P.t) {
+          rk = __ldcg(row);
+          rl = __ldcg(row + 1);
+        }
+        top_t_merge(rk, rl, nb_k, nb_l, P.t, G.lane);
+        if (G.lane < P.t) {
+          __stcg(row, rk);
+          __stcg(row + 1, rl);
+        }
+      }
     }
     finish();
 #ifdef PF_TIMELINE
@@ -1392,50 +1422,6 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
       }
     }
 #endif
-  }
-
-  // ---- All-to-All t >= 2: the CTA's best t of its groups' lists -> pool_cta
-  //      (the stage buffers are free: no load is in flight after the loop)
-  if (P.pool_cta) {
-    u64* lists = reinterpret_cast<u64*>(gs + C::g_stage);   // this group's [t] keys, then [t] entries
-    if (G.wig == 0 && G.lane < P.t) {
-      lists[G.lane] = gtop_k;
-      lists[P.t + G.lane] = gtop_l;
-    }
-    __syncthreads();
-    if (threadIdx.x < 32) {
-      // candidate i = group i / t, item i % t; S * t <= 15 * 32
-      u64 ck = 0ull, cl = 0ull;
-      for (int r = 0; r < P.t; ++r) {
-        u64 mine = 0ull;
-        int mi = -1;
-        for (int i = threadIdx.x; i < C::S * P.t; i += 32) {
-          const int gg = i / P.t, jj = i - gg * P.t;
-          const u64 kk = reinterpret_cast<u64*>(smem + C::c_groups + gg * C::group_bytes + C::g_stage)[jj];
-          if (kk > mine) {
-            mine = kk;
-            mi = i;
-          }
-        }
-        const u64 w = warp_max_u64(mine);
-        if (w != 0ull && mine == w) {   // unique owner (keys carry the particle index)
-          const int gg = mi / P.t, jj = mi - gg * P.t;
-          u64* gl = reinterpret_cast<u64*>(smem + C::c_groups + gg * C::group_bytes + C::g_stage);
-          ck = w;
-          cl = gl[P.t + jj];
-          gl[jj] = 0ull;
-        }
-        __syncwarp();
-        const int owner = __ffs(__ballot_sync(0xFFFFFFFFu, w != 0ull && mine == w)) - 1;
-        const u64 wl = owner >= 0 ? __shfl_sync(0xFFFFFFFFu, cl, owner) : 0ull;
-        if (threadIdx.x == 0) {
-          P.pool_cta[(static_cast<long long>(blockIdx.x) * P.tt + r) * 2] = w;
-          P.pool_cta[(static_cast<long long>(blockIdx.x) * P.tt + r) * 2 + 1] = wl;
-        }
-        __syncwarp();
-      }
-      (void)ck;
-    }
   }
 
   // ---- a5: the last CTA to finish copies the winning particle (R6)
@@ -1494,10 +1480,11 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
           pool[0] = unord_f32(static_cast<uint32_t>(key >> 32));
           pool[1] = __uint_as_float(gidx);
         }
-      } else if (P.pool_cta) {
-        pool_top_t_cta<E>(P, pool);
       } else {
-        pool_top_t<E>(P, P.mb_cur, P.n_local * P.t, pool);
+        // reduction scratch: group 0's stage buffer (no load in flight after the loop)
+        u64* red = reinterpret_cast<u64*>(smem + C::c_groups + C::g_stage);
+        if (P.pool_cta) pool_top_t_cta<E>(P, pool, red, static_cast<long long>(gridDim.x) * C::S);
+        else pool_top_t<E>(P, P.mb_cur, P.n_local * P.t, pool, red);
       }
     }
     if (tid == 0) {

@@ -220,11 +220,11 @@ float* mailbox_parity(pf_handle* h, long long k) {
   return h->mailbox + (k & 1) * h->g.n_ext * h->g.tt * h->g.E;
 }
 
-// All-to-All with t >= 2: per-CTA best-t candidates after the mailbox parities
-// ({order key, entry} u64 pairs for up to kPoolCtas CTAs of the step kernel).
-constexpr long long kPoolCtas = 8192;
+// All-to-All with t >= 2: per-group best-t candidates after the mailbox parities
+// ({order key, entry} u64 pairs for up to kPoolGroups groups of the step kernel).
+constexpr long long kPoolGroups = 16384;
 size_t pool_cta_bytes(const pf_config* cfg, const Geometry& g) {
-  return (!g.central && cfg->topo == PF_TOPO_ALL2ALL && cfg->t >= 2) ? sizeof(u64) * 2 * kPoolCtas * g.tt : 0;
+  return (!g.central && cfg->topo == PF_TOPO_ALL2ALL && cfg->t >= 2) ? sizeof(u64) * 2 * kPoolGroups * g.tt : 0;
 }
 
 // Host-input steps of a single-rank filter stream their estimate record into
@@ -549,7 +549,8 @@ pf_status pf_init(const pf_config* cfg, const pf_model_params* model, const pf_b
     const long long ctas_needed = (g.n_local + h->ke->s - 1) / h->ke->s;
     const long long grid = static_cast<long long>(bps) * sms;
     h->grid = static_cast<int>(grid < ctas_needed ? grid : ctas_needed);
-    if (pool_cta_bytes(cfg, g) && h->grid > kPoolCtas) h->grid = static_cast<int>(kPoolCtas);
+    if (pool_cta_bytes(cfg, g) && static_cast<long long>(h->grid) * h->ke->s > kPoolGroups)
+      h->grid = static_cast<int>(kPoolGroups / h->ke->s);
   }
   // scratch: zero keys / counter; prior parameters
   float prior[128];

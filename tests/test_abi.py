@@ -65,9 +65,9 @@ def test_query_sizes(B):
     s2 = B.pf_query_sizes(_cfg(B, world=4, rank=1, t=2), _model(B, 5))
     assert s2.state == 4 * 10 * 4 * 64
     assert s2.mailbox == 4 * 2 * (4 + 2) * 2 * 11
-    # All-to-All, t = 2: one pool row, then the per-CTA best-t candidates (8192 CTAs x t x 16 B)
+    # All-to-All, t = 2: one pool row, then the per-group best-t candidates (16384 groups x t x 16 B)
     s3 = B.pf_query_sizes(_cfg(B, topo=B.PF_TOPO_ALL2ALL, t=2), _model(B, 2))
-    assert s3.mailbox == 4 * 2 * (16 + 1) * 2 * (d + 2) + 16 * 8192 * 2
+    assert s3.mailbox == 4 * 2 * (16 + 1) * 2 * (d + 2) + 16 * 16384 * 2
 
 
 @pytest.mark.parametrize("kw,code", [
