@@ -5,5 +5,5 @@ cd "${GRAFT_REPO_ROOT:-.}"
 mkdir -p gpurun_out
 bash scripts/profile_round.sh
 timeout 300 python bench.py --impl reference --steps 10 --warmup 3 > gpurun_out/bench_reference.json 2> gpurun_out/bench_reference.err
-timeout 900 python scripts/sanitize_run.py > gpurun_out/sanitizer.txt 2>&1
+bash scripts/gcall_sanitize.sh
 ls -la gpurun_out
