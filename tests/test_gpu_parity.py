@@ -331,3 +331,39 @@ def test_error_behaviour(P, W):
     assert B.pf_last_error(g.h) == B.PF_OK
     with pytest.raises(B.PFError):
         P.ParticleFilter(tr["mu0"], tr["sigma0"], P.ArmModel(n_joints=3), m=64, n_filters=4)   # not compiled
+
+
+@pytest.mark.parametrize("central", [False, True])
+def test_device_inputs_streamed_and_batched(P, orc, W, central):
+    """Device-resident inputs (the bench's timed path): per-step pf_step +
+    pf_estimate (record copied from the device) and pf_step_batch (records
+    written on the device) both equal the oracle's estimates, step by step."""
+    import torch
+    nj, T = 5, 8
+    m, N = (8192, 1) if central else (64, 16)
+    topo, t = ("none", 0) if central else ("ring", 1)
+    tr = W.make_trajectory(nj, T, 3)
+    kw = dict(m=m, n_filters=N, t=t, topo=topo, resampler="rws", seed=5)
+    zs = torch.tensor(tr["Z"][1:T + 1], device="cuda")
+    us = torch.tensor(tr["U"][:T], device="cuda")
+    g = P.ParticleFilter(tr["mu0"], tr["sigma0"], P.ArmModel(n_joints=nj), device_inputs=True, **kw)
+    gb = P.ParticleFilter(tr["mu0"], tr["sigma0"], P.ArmModel(n_joints=nj), device_inputs=True, **kw)
+    o = orc.Filter(orc.Config(**kw), orc.Model(n_joints=nj), tr["mu0"], tr["sigma0"])
+    d = nj + 4
+    est = torch.zeros(T, 4 + d, device="cuda")
+    gb.step_batch(zs, us, est)
+    est = est.cpu().numpy()
+    for k in range(1, T + 1):
+        g.step(zs[k - 1], us[k - 1])
+        o.step(tr["Z"][k], tr["U"][k - 1])
+        xg, lg, ig = g.estimate()
+        xo, lo, io = o.estimate()
+        assert ig == io, (k, ig, io)
+        np.testing.assert_array_equal(xg, xo)
+        np.testing.assert_array_equal(est[k - 1, 4:], xo)
+        assert est[k - 1, 2] == np.float32(lo)
+    xb, _, ib = gb.estimate()
+    assert ib == io
+    np.testing.assert_array_equal(xb, xo)
+    g.close()
+    gb.close()
