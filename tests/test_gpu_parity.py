@@ -136,6 +136,10 @@ def test_full_filter_c1(P, orc, W):
     (5, 1024, 4, 4, "torus", "rws"),
     (5, 64, 16, 2, "all2all", "vose"),
     (2, 256, 64, 1, "all2all", "rws"),
+    # more sub-filters than resident groups: groups merge several sub-filters'
+    # best t into their running pool candidates (All-to-All, t >= 2)
+    (5, 32, 8192, 2, "all2all", "rws"),
+    (5, 32, 8192, 4, "all2all", "vose"),
 ])
 def test_full_filter_variants(P, orc, W, nj, m, N, t, topo, res):
     _run_compare(P, orc, W, nj, m, N, 12, t=t, topo=topo, res=res, seed=nj * 1000 + m)
