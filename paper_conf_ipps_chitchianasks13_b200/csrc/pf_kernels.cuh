@@ -141,8 +141,8 @@ __device__ __forceinline__ unsigned long long tl_now() {
 // group; the per-particle sample/weight loop over a thread's P slots is
 // unrolled UNR times (P for full unrolling; 1 keeps one copy of the
 // ~10–40 KB per-particle code in the instruction cache).
-#ifndef PF_ROLL_MIN_D
-#define PF_ROLL_MIN_D 16
+#ifndef PF_CHUNK_MIN_D
+#define PF_CHUNK_MIN_D 16
 #endif
 #ifndef PF_X2_DEFAULT
 #define PF_X2_DEFAULT 1
@@ -164,7 +164,7 @@ struct KCfg {
   // large states (the high-DOF arm): the joint chain runs as a loop over
   // chunks of four joints instead of being unrolled d times, so the
   // per-particle code fits the instruction cache (ncu: no_instruction stalls)
-  static constexpr bool ROLLED = D > PF_ROLL_MIN_D;
+  static constexpr bool CHUNKED = D > PF_CHUNK_MIN_D;
   static_assert(P >= 1 && P * T == M, "M must be a multiple of the group size");
   static_assert(P <= 32, "exclusion masks are 32-bit");
   static_assert(S >= 1 && S <= 15, "named barriers 1..S");
@@ -266,53 +266,6 @@ __device__ __forceinline__ X warp_incl_scan(X x, int lane) {
   return x;
 }
 
-// Slot-order inclusive prefix of per-slot values val[P] over the group
-// (strided slots, KCfg::slot): out[j] = sum of val over slots <= slot(t, j).
-// Returns the group total.  One group barrier when GW > 1.
-template <class C, typename X>
-__device__ __forceinline__ X slot_scan_incl(const X (&val)[C::P], X (&out)[C::P], GroupCtx& G) {
-  constexpr int P = C::P, GW = C::GW;
-  X w[P];
-#pragma unroll
-  for (int j = 0; j < P; ++j) w[j] = val[j];
-#pragma unroll
-  for (int o = 1; o < 32; o <<= 1) {
-#pragma unroll
-    for (int j = 0; j < P; ++j) {
-      const X y = __shfl_up_sync(0xFFFFFFFFu, w[j], o);
-      if (G.lane >= o) w[j] += y;
-    }
-  }
-  if constexpr (GW == 1) {
-    X base = 0;
-#pragma unroll
-    for (int j = 0; j < P; ++j) {
-      out[j] = base + w[j];
-      base += __shfl_sync(0xFFFFFFFFu, w[j], 31);
-    }
-    return base;
-  } else {
-    X* r = reinterpret_cast<X*>(G.red + G.rb * 32);
-    G.rb ^= 1;
-    if (G.lane == 31) {
-#pragma unroll
-      for (int j = 0; j < P; ++j) r[j * GW + G.wig] = w[j];
-    }
-    gsync<GW>(G.g);
-    X run = 0;
-#pragma unroll
-    for (int j = 0; j < P; ++j) {
-#pragma unroll
-      for (int ww = 0; ww < GW; ++ww) {
-        const X v = r[j * GW + ww];
-        if (ww == G.wig) out[j] = run + w[j];
-        run += v;
-      }
-    }
-    return run;
-  }
-}
-
 // P contiguous elements <-> registers with the widest shared-memory vectors
 template <typename X, int P>
 __device__ __forceinline__ void vload(const X* src, X (&v)[P]) {
@@ -346,7 +299,7 @@ __device__ __forceinline__ void vstore(X* dst, const X (&v)[P]) {
 // Slot-order inclusive prefix through shared memory: the strided per-thread
 // values are transposed (buf[slot]), thread t scans the P contiguous slots
 // [tP, tP + P) serially, ONE warp shuffle scan of the per-thread totals (plus
-// one cross-warp level) replaces the P shuffle scans of slot_scan_incl, and
+// one cross-warp level) instead of one shuffle scan per slot chunk, and
 // buf[s] ends up holding the inclusive prefix of every slot s (slot order).
 // Returns the group total.  Group barriers: 2 (+1 when GW > 1).
 template <class C, typename X>
@@ -385,35 +338,6 @@ __device__ __forceinline__ X slot_scan_smem(const X (&val)[C::P], X* buf, GroupC
   vstore<X, P>(buf + G.t * P, v);
   gsync<GW>(G.g);
   return total;
-}
-
-// first index i in [0, n) with a[i] >= x
-__device__ __forceinline__ int lower_bound_u64(const u64* a, int n, u64 x) {
-  int lo = 0;
-  while (n > 0) {
-    const int half = n >> 1;
-    if (a[lo + half] < x) {
-      lo += half + 1;
-      n -= half + 1;
-    } else {
-      n = half;
-    }
-  }
-  return lo;
-}
-// first index i in [0, n) with a[i] > x
-__device__ __forceinline__ int upper_bound_u64(const u64* a, int n, u64 x) {
-  int lo = 0;
-  while (n > 0) {
-    const int half = n >> 1;
-    if (a[lo + half] <= x) {
-      lo += half + 1;
-      n -= half + 1;
-    } else {
-      n = half;
-    }
-  }
-  return lo;
 }
 
 // One level of the RWS binary search over u32 inclusive sums in shared
@@ -1285,7 +1209,7 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
           outa[c * M] = lo2(v);
           outb[c * M] = hi2(v);
         };
-        if constexpr (C::ROLLED) {
+        if constexpr (C::CHUNKED) {
           SampleChunked2<NJ>::run(P.mc2, hsu2_s, z2_s, x, gen, A, store2);
         } else {
           SampleStream2<NJ, 0>::run(P.mc2, hsu2_s, z2_s, x, gen, A, store2);
