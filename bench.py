@@ -190,10 +190,13 @@ def run_ours(a) -> None:
     zs = torch.tensor(tr["Z"][1:], device=dev)
     us = torch.tensor(tr["U"][:-1], device=dev)
 
+    transport = {"p2p": False}   # multi-rank: halo + estimate inside the kernel (peer transport) or NCCL
+
     # ---- device-resident inputs (value) -----------------------------------
     def device_run(resampler: str, flush_l2: bool, steps: int):
         pf = F.ParticleFilter(tr["mu0"], tr["sigma0"], model, resampler=resampler, device_inputs=True, **kw)
         df = Dd.DistributedFilter(pf)
+        transport["p2p"] = df.p2p
         stream = pf.stream
         for k in range(Wm):
             df.step(zs[k], us[k])
@@ -305,7 +308,10 @@ def run_ours(a) -> None:
             "e2e": {"value": e2e_value, "unit": "particle-steps/s", "estimates_per_s": 1e3 / e2e_ms,
                     "ms_per_step": e2e_ms, "h2d_bytes_per_step": 4 * (NJ + 2 + NJ),
                     "d2h_bytes_per_step": 4 * (4 + D)},
-            "clocks": clocks, "gpu_launches": K * (1 if world == 1 else 2), **extras}
+            "clocks": clocks, "gpu_launches": K * (1 if (world == 1 or transport["p2p"]) else 2), **extras}
+    if world > 1:
+        line["config"]["transport"] = ("nvlink peer stores + device rendezvous in the step kernel" if transport["p2p"]
+                                       else "nccl send/recv halos + all-gather of records")
     if rank == 0 and world == 1:
         rate, nsteps, particles, times = _oracle_rate(a.cpu_seconds)
         line["cpu_baseline"] = {"value": rate, "unit": "particle-steps/s", "cores": 1, "kind": "oracle",

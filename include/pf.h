@@ -290,6 +290,39 @@ pf_status pf_debug_math(int32_t fn, const uint32_t* in, uint32_t* out, int64_t n
  * kernels' branch-free sqrt differs from IEEE sqrt.rn (exhaustive, on device). */
 pf_status pf_debug_check_sqrt(uint32_t lo_bits, uint32_t hi_bits, uint64_t* mismatches);
 
+/* ---- Peer transport (multi-rank on one node) -------------
+ * The exchange halo (Alg.2 l.10–14; "exchanged particles are
+ * unique to neighbor pairs", §VI-E) and the global estimate (the
+ * particle with the highest global weight, :16 §IV / :20 §VI-D) cross ranks
+ * inside the step kernel itself, over NVLink / NVSwitch peer memory, instead of
+ * NCCL send/recv + all-gather + pf_reduce_records around it:
+ *  - the reduce phase writes each boundary sub-filter's best-t entries straight
+ *    into the neighbour ranks' halo rows (the pf_shard layout: ring — local
+ *    sub-filter 0 -> rank r-1's row n_local+1, the last -> rank r+1's row
+ *    n_local; torus — the first grid row -> rank r-1's rows n_local+C.., the
+ *    last -> rank r+1's rows n_local..);
+ *  - the last CTA writes the shard's best record into every rank's peer block,
+ *    raises its step flag there (system-scope release) and waits for every
+ *    rank's flag (acquire): a device-side rendezvous per step, after which the
+ *    exact max over the world records is the global estimate on every rank.
+ * Ring and 2D torus, world 2..8, steps strictly increasing after connecting.
+ * pf_peer_export: this rank's blob (CUDA IPC handles of the caller's mailbox
+ *   allocation + offset, and of a 4 KiB runtime-owned peer block; the rank).
+ *   Host blob[PF_PEER_BLOB_BYTES].  Call before the first step.
+ * pf_peer_connect: blobs [world][PF_PEER_BLOB_BYTES] of all ranks in rank order
+ *   (e.g. all-gathered through torch.distributed); opens the peers' blocks and
+ *   the neighbours' mailboxes (cudaIpcOpenMemHandle, lazy peer access).
+ * pf_peer_connect_local: the same for `world` handles of ONE process (tests on
+ *   one device; their steps must run on different streams).
+ * Errors: PF_ESTATE (world == 1, central filter, already stepped / connected,
+ *   export missing), PF_EUNSUPPORTED (All-to-All: its pool keeps the NCCL path),
+ *   PF_ECUDA (IPC failure; the handle stays on the NCCL path). */
+#define PF_PEER_BLOB_BYTES 160
+pf_status pf_peer_export(pf_handle* h, uint8_t* blob);
+pf_status pf_peer_connect(pf_handle* h, const uint8_t* blobs);
+pf_status pf_peer_connect_local(pf_handle* const* handles, int32_t world);
+int32_t pf_peer_connected(const pf_handle* h);
+
 /* Release host metadata; NULL-safe.  Does not free caller buffers. */
 pf_status pf_destroy(pf_handle* h);
 

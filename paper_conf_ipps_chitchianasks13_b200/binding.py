@@ -25,7 +25,7 @@ ENTRY_POINTS = [
     "pf_reduce_records", "pf_reduce_pool", "pf_get_shard", "pf_get_particles", "pf_set_particles", "pf_debug_sample_weight",
     "pf_debug_resample", "pf_debug_exchange", "pf_set_trace", "pf_get_trace", "pf_destroy", "pf_strerror",
     "pf_last_error", "pf_supported", "pf_debug_math", "pf_debug_check_sqrt", "pf_estimate_mean", "pf_mean_partial",
-    "pf_reduce_means",
+    "pf_reduce_means", "pf_peer_export", "pf_peer_connect", "pf_peer_connect_local", "pf_peer_connected",
 ]
 PF_MATH = {"sin": 0, "cos": 1, "log": 2, "expq": 3, "sqrt": 4, "sincos2pi": 5, "normal_pair": 6, "philox": 7}
 
@@ -108,6 +108,13 @@ def lib() -> C.CDLL:
         L.pf_debug_math.restype = ST
         L.pf_debug_check_sqrt.argtypes = [C.c_uint32, C.c_uint32, P]
         L.pf_debug_check_sqrt.restype = ST
+        if hasattr(L, "pf_peer_export"):   # (dev A/B builds of older sources lack the peer transport)
+            for name, args in {"pf_peer_export": [P, P], "pf_peer_connect": [P, P],
+                               "pf_peer_connect_local": [P, I32]}.items():
+                getattr(L, name).argtypes = args
+                getattr(L, name).restype = ST
+            L.pf_peer_connected.argtypes = [P]
+            L.pf_peer_connected.restype = I32
         _lib = L
     return _lib
 
@@ -258,3 +265,26 @@ def pf_debug_check_sqrt(lo_bits: int, hi_bits: int) -> int:
     bad = C.c_uint64()
     check(lib().pf_debug_check_sqrt(lo_bits, hi_bits, C.byref(bad)), "pf_debug_check_sqrt")
     return bad.value
+
+
+PF_PEER_BLOB_BYTES = 160
+
+
+def pf_peer_export(h) -> bytes:
+    buf = (C.c_uint8 * PF_PEER_BLOB_BYTES)()
+    check(lib().pf_peer_export(h, buf), "pf_peer_export")
+    return bytes(buf)
+
+
+def pf_peer_connect(h, blobs: bytes) -> None:
+    buf = (C.c_uint8 * len(blobs)).from_buffer_copy(blobs)
+    check(lib().pf_peer_connect(h, buf), "pf_peer_connect")
+
+
+def pf_peer_connect_local(handles) -> None:
+    arr = (C.c_void_p * len(handles))(*[h.value for h in handles])
+    check(lib().pf_peer_connect_local(arr, len(handles)), "pf_peer_connect_local")
+
+
+def pf_peer_connected(h) -> bool:
+    return bool(lib().pf_peer_connected(h))

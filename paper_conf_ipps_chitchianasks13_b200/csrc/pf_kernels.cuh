@@ -48,6 +48,12 @@ enum : int { POLICY_ALWAYS = 0, POLICY_ESS = 1, POLICY_FREQ = 2 };
 // polls it instead of synchronizing the stream)
 constexpr int kRecordSeq = 127;
 
+// Peer transport (world > 1 on one node, NVLink/NVSwitch peer memory): every
+// rank's runtime owns a small "peer block" that the other ranks write into:
+// [kMaxRanks] u64 step flags, then [kMaxRanks][kPeerRec] float records.
+constexpr int kMaxRanks = 8;
+constexpr int kPeerRec = 40;   // 4 + d <= 36 floats, padded
+
 struct StepParams {
   ArmConsts mc;
   ArmConsts2 mc2;          // mc with every field duplicated (packed f32x2 operands)
@@ -77,6 +83,13 @@ struct StepParams {
   int policy;              // R21: POLICY_ALWAYS / _ESS / _FREQ
   unsigned long long policy_param;   // ESS: tau 2^16; FREQ: threshold on a Philox word
   uint32_t rk[20];         // Philox round keys (key0 + r W0, key1 + r W1), r = 0..9
+  // peer transport (nullable peer_mb[0] = off): the prev / next neighbour
+  // rank's mailbox base (ring: r -1 / r + 1; torus: the rank above / below),
+  // every rank's peer block (own included), this rank and the world size
+  float* peer_mb[2];
+  unsigned char* peer_blk[kMaxRanks];
+  int rank, world;
+  long long mb_parity;     // floats per mailbox parity (n_ext * tt * E), same on every rank
   float zin[32];           // step inputs carried by the launch itself (host-input mode)
   float uin[32];
 };
@@ -702,6 +715,40 @@ struct SampleChunked2 {
     SampleStream2<NJ, 1 + 2 * NC>::run(mc, hsu2, z2, x, gen, A, out);
   }
 };
+
+// Peer transport, halo rows (reading R3/R4 and the halo plan of
+// distributed.py): ring — local sub-filter 0 -> the previous rank's row
+// n_local + 1, the last -> the next rank's row n_local; torus — the first grid
+// row -> the rank above, rows n_local + C + c, the last grid row -> the rank
+// below, rows n_local + c.  The row's first t entries [logw, index bits, x],
+// copied by one warp (out of line: no register cost in the step loop).
+template <int E>
+__device__ __noinline__ void peer_halo_copy(const StepParams& P, long long n, int lane) {
+  const long long nl = P.n_local, par = static_cast<long long>(P.k & 1u) * P.mb_parity;
+  long long row0 = -1, row1 = -1;   // destination rows in the previous / next rank
+  if (P.topo == TOPO_RING) {
+    if (n == 0) row0 = nl + 1;
+    if (n == nl - 1) row1 = nl;
+  } else {
+    const long long Cc = P.C, lr = n / Cc, c = n - lr * Cc, rows = nl / Cc;
+    if (lr == 0) row0 = nl + Cc + c;
+    if (lr == rows - 1) row1 = nl + c;
+  }
+  if (row0 < 0 && row1 < 0) return;
+  const float* src = P.mb_cur + n * P.tt * E;   // the row's first t entries
+  for (int e = lane; e < P.t * E; e += 32) {
+    const float v = __ldcg(src + e);
+    if (row0 >= 0) P.peer_mb[0][par + row0 * P.tt * E + e] = v;
+    if (row1 >= 0) P.peer_mb[1][par + row1 * P.tt * E + e] = v;
+  }
+}
+
+__device__ __forceinline__ unsigned long long* peer_flags(unsigned char* blk) {
+  return reinterpret_cast<unsigned long long*>(blk);
+}
+__device__ __forceinline__ float* peer_rec(unsigned char* blk, int r) {
+  return reinterpret_cast<float*>(blk + sizeof(unsigned long long) * kMaxRanks) + r * kPeerRec;
+}
 
 // Best t of the union of two descending lists held by lanes 0..t-1 (run list
 // r, new list nb; keys unique or 0 = empty) into r, by t rounds of warp max.
@@ -1332,6 +1379,10 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
       }
     }
     finish();
+    // peer transport: a boundary sub-filter's best-t row (complete in this
+    // rank's mailbox after finish()'s group barrier) also goes straight into
+    // the neighbour rank's halo row (NVLink stores)
+    if (P.peer_mb[0] && (mode == MODE_STEP || mode == MODE_PUBLISH) && G.wig == 0) peer_halo_copy<E>(P, n, G.lane);
 #ifdef PF_TIMELINE
     if (G.t == 0) {
       const unsigned long long tl_end = tl_now();
@@ -1357,7 +1408,8 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
   if (threadIdx.x == 0) {
     // the CTA barrier orders every thread's writes (mailbox rows, key) before
     // thread 0's cumulative gpu-scope fence and the completion count
-    __threadfence();
+    if (P.peer_mb[0]) __threadfence_system();   // this CTA's peer halo stores before the count
+    else __threadfence();
     const unsigned int prev = atomicAdd(P.counter, 1u);
     s_last = (prev == gridDim.x - 1) ? 1u : 0u;
   }
@@ -1371,20 +1423,65 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
       const long long col = static_cast<long long>(gidx) - P.g0 * M;
       const float* blk = P.parts + (col / M) * C::ROW + (col % M);
       float* outs[3] = {P.record, P.est_out, P.record_host};
-      if (tid < D) {
-        const float v = __ldcg(blk + tid * M);
+      if (P.peer_mb[0] && (mode == MODE_STEP || mode == MODE_PUBLISH)) {
+        // peer transport: this shard's best record into slot `rank` of every
+        // rank's peer block, then step flags, then wait for every rank's flag
+        // (device-side rendezvous over NVLink), then the exact max over the
+        // world records (the all-gather + pf_reduce_records of the NCCL path)
+        if (tid < D) {
+          const float v = __ldcg(blk + tid * M);
+          for (int r = 0; r < P.world; ++r) peer_rec(P.peer_blk[r], P.rank)[4 + tid] = v;
+        }
+        if (tid == 0) {
+          const float r4[4] = {__uint_as_float(static_cast<uint32_t>(key)),
+                               __uint_as_float(static_cast<uint32_t>(key >> 32)),
+                               unord_f32(static_cast<uint32_t>(key >> 32)), 0.0f};
+          for (int r = 0; r < P.world; ++r)
+            for (int c = 0; c < 4; ++c) peer_rec(P.peer_blk[r], P.rank)[c] = r4[c];
+        }
+        __threadfence_system();
+        __syncthreads();
+        const unsigned long long kk = P.k;
+        if (tid < P.world) {
+          unsigned long long* f = peer_flags(P.peer_blk[tid]) + P.rank;
+          asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(f), "l"(kk) : "memory");
+          const unsigned long long* mine = peer_flags(P.peer_blk[P.rank]) + tid;
+          unsigned long long seen;
+          do {
+            asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(seen) : "l"(mine) : "memory");
+          } while (seen < kk);
+        }
+        __syncthreads();
+        if (tid < 32) {
+          const float* rec0 = peer_rec(P.peer_blk[P.rank], 0);
+          u64 k2 = 0ull;
+          if (tid < P.world)
+            k2 = static_cast<u64>(__float_as_uint(__ldcv(rec0 + tid * kPeerRec))) |
+                 (static_cast<u64>(__float_as_uint(__ldcv(rec0 + tid * kPeerRec + 1))) << 32);
+          const u64 w = warp_max_u64(k2);
+          const int src = __ffs(__ballot_sync(0xFFFFFFFFu, tid < P.world && k2 == w)) - 1;
+          for (int c = tid; c < 4 + D; c += 32) {
+            const float v = __ldcv(rec0 + src * kPeerRec + c);
+            for (int o = 0; o < 3; ++o)
+              if (outs[o]) outs[o][c] = v;
+          }
+        }
+      } else {
+        if (tid < D) {
+          const float v = __ldcg(blk + tid * M);
 #pragma unroll
-        for (int o = 0; o < 3; ++o)
-          if (outs[o]) outs[o][4 + tid] = v;
-      }
-      if (tid == 0) {
-        const float r[4] = {__uint_as_float(static_cast<uint32_t>(key)), __uint_as_float(static_cast<uint32_t>(key >> 32)),
-                            unord_f32(static_cast<uint32_t>(key >> 32)), 0.0f};
+          for (int o = 0; o < 3; ++o)
+            if (outs[o]) outs[o][4 + tid] = v;
+        }
+        if (tid == 0) {
+          const float r[4] = {__uint_as_float(static_cast<uint32_t>(key)), __uint_as_float(static_cast<uint32_t>(key >> 32)),
+                              unord_f32(static_cast<uint32_t>(key >> 32)), 0.0f};
 #pragma unroll
-        for (int o = 0; o < 3; ++o)
-          if (outs[o])
+          for (int o = 0; o < 3; ++o)
+            if (outs[o])
 #pragma unroll
-            for (int c = 0; c < 4; ++c) outs[o][c] = r[c];
+              for (int c = 0; c < 4; ++c) outs[o][c] = r[c];
+        }
       }
       if (P.record_host) {   // completion word polled by pf_estimate (after the record, system scope)
         __threadfence_system();

@@ -198,6 +198,14 @@ struct pf_handle {
   bool trace;
   long long* d_src;
   int* d_anc;
+  // peer transport (pf_peer_connect*): the neighbour ranks' mailboxes and every
+  // rank's peer block (flags + records), this rank's own block (cudaMalloc'd)
+  bool peers;
+  float* peer_mb[2];
+  unsigned char* peer_blk[pf::kMaxRanks];
+  unsigned char* own_blk;
+  void* opened[2 * pf::kMaxRanks];   // IPC mappings to close
+  int n_opened;
   bool mapped;         // PF_NO_MAPPED unset at init
   bool last_mapped;    // the last step wrote its record (and step number) into rec_host
   float* rec_host;     // mapped pinned host floats: [0, 4+d) estimate record, [48, 48+d) weighted mean
@@ -231,7 +239,7 @@ size_t pool_cta_bytes(const pf_config* cfg, const Geometry& g) {
 // mapped pinned host memory (pf_estimate polls it); device-input steps keep it
 // on the device (record / est_out) and pf_estimate copies it on demand.
 bool streams_record(const pf_handle* h) {
-  return h->mapped && !(h->cfg.flags & PF_DEVICE_INPUTS) && h->cfg.world == 1;
+  return h->mapped && !(h->cfg.flags & PF_DEVICE_INPUTS) && (h->cfg.world == 1 || h->peers);
 }
 
 pf::StepParams base_params(pf_handle* h, long long k, int mode) {
@@ -266,6 +274,14 @@ pf::StepParams base_params(pf_handle* h, long long k, int mode) {
   p.C = h->g.C;
   p.pool_row = h->g.n_local + (h->cfg.world > 1 ? h->cfg.world : 0);
   p.pool_local_row = h->g.n_local + (h->cfg.world > 1 ? h->cfg.rank : 0);
+  if (h->peers) {
+    p.peer_mb[0] = h->peer_mb[0];
+    p.peer_mb[1] = h->peer_mb[1];
+    for (int r = 0; r < pf::kMaxRanks; ++r) p.peer_blk[r] = h->peer_blk[r];
+  }
+  p.rank = h->cfg.rank;
+  p.world = h->cfg.world;
+  p.mb_parity = h->g.n_ext * h->g.tt * h->g.E;
   p.pool_cta = pool_cta_bytes(&h->cfg, h->g)
                    ? reinterpret_cast<u64*>(h->mailbox + 2 * h->g.n_ext * h->g.tt * h->g.E)
                    : nullptr;
@@ -946,9 +962,132 @@ pf_status pf_get_trace(pf_handle* h, int64_t* src, int32_t* ancestors) {
   return sticky(h, e);
 }
 
+// ---- peer transport (NVLink / NVSwitch peer memory via CUDA IPC) ----------
+namespace {
+constexpr size_t kPeerBlockBytes = 4096;   // [kMaxRanks] u64 flags + [kMaxRanks][kPeerRec] floats
+static_assert(sizeof(u64) * pf::kMaxRanks + sizeof(float) * pf::kMaxRanks * pf::kPeerRec <= kPeerBlockBytes, "");
+
+pf_status peer_check(const pf_handle* h) {
+  if (!h) return PF_EINVAL;
+  if (h->err != PF_OK) return h->err;
+  if (h->g.central || h->cfg.world < 2 || h->cfg.world > pf::kMaxRanks) return PF_ESTATE;
+  if (h->cfg.topo != PF_TOPO_RING && h->cfg.topo != PF_TOPO_TORUS2D) return PF_EUNSUPPORTED;
+  if (h->step != 0 || h->peers) return PF_ESTATE;   // connect once, before the first step
+  return PF_OK;
+}
+pf_status ensure_block(pf_handle* h) {
+  if (h->own_blk) return PF_OK;
+  cudaError_t e = cudaMalloc(&h->own_blk, kPeerBlockBytes);
+  if (e == cudaSuccess) e = cudaMemset(h->own_blk, 0, kPeerBlockBytes);
+  if (e != cudaSuccess) {
+    h->own_blk = nullptr;
+    return sticky(h, e);
+  }
+  return PF_OK;
+}
+void set_peers(pf_handle* h, float* prev_mb, float* next_mb, unsigned char* const* blks) {
+  h->peer_mb[0] = prev_mb;
+  h->peer_mb[1] = next_mb;
+  for (int r = 0; r < pf::kMaxRanks; ++r) h->peer_blk[r] = r < h->cfg.world ? blks[r] : nullptr;
+  h->peers = true;
+}
+}  // namespace
+
+pf_status pf_peer_export(pf_handle* h, uint8_t* blob) {
+  pf_status st = peer_check(h);
+  if (st != PF_OK || !blob) return st != PF_OK ? st : PF_EINVAL;
+  if ((st = ensure_block(h)) != PF_OK) return st;
+  // the caller's mailbox lives inside some cudaMalloc allocation: export that
+  // allocation and the mailbox's offset in it
+  typedef int (*AddrRange)(unsigned long long*, size_t*, unsigned long long);
+  void* fn = nullptr;
+  cudaDriverEntryPointQueryResult q;
+  cudaError_t e = cudaGetDriverEntryPoint("cuMemGetAddressRange", &fn, cudaEnableDefault, &q);
+  if (e != cudaSuccess || !fn) return sticky(h, e != cudaSuccess ? e : cudaErrorNotSupported);
+  unsigned long long base = 0;
+  size_t size = 0;
+  if (reinterpret_cast<AddrRange>(fn)(&base, &size, reinterpret_cast<unsigned long long>(h->mailbox)) != 0)
+    return sticky(h, cudaErrorInvalidValue);
+  cudaIpcMemHandle_t hm, hb;
+  e = cudaIpcGetMemHandle(&hm, reinterpret_cast<void*>(base));
+  if (e == cudaSuccess) e = cudaIpcGetMemHandle(&hb, h->own_blk);
+  if (e != cudaSuccess) return sticky(h, e);
+  const unsigned long long off = reinterpret_cast<unsigned long long>(h->mailbox) - base;
+  std::memset(blob, 0, PF_PEER_BLOB_BYTES);
+  std::memcpy(blob, &hm, sizeof(hm));
+  std::memcpy(blob + 64, &off, sizeof(off));
+  std::memcpy(blob + 72, &hb, sizeof(hb));
+  const int64_t rank = h->cfg.rank;
+  std::memcpy(blob + 136, &rank, sizeof(rank));
+  return PF_OK;
+}
+
+pf_status pf_peer_connect(pf_handle* h, const uint8_t* blobs) {
+  pf_status st = peer_check(h);
+  if (st != PF_OK || !blobs) return st != PF_OK ? st : PF_EINVAL;
+  if (!h->own_blk) return PF_ESTATE;   // pf_peer_export first
+  const int W = h->cfg.world, r = h->cfg.rank;
+  const int prev = (r + W - 1) % W, next = (r + 1) % W;
+  unsigned char* blks[pf::kMaxRanks] = {};
+  float* mbs[pf::kMaxRanks] = {};
+  for (int q = 0; q < W; ++q) {
+    const uint8_t* b = blobs + static_cast<size_t>(q) * PF_PEER_BLOB_BYTES;
+    int64_t qr;
+    std::memcpy(&qr, b + 136, sizeof(qr));
+    if (qr != q) return PF_EINVAL;
+    if (q == r) {
+      blks[q] = h->own_blk;
+      mbs[q] = h->mailbox;
+      continue;
+    }
+    cudaIpcMemHandle_t hb;
+    std::memcpy(&hb, b + 72, sizeof(hb));
+    void* pb = nullptr;
+    cudaError_t e = cudaIpcOpenMemHandle(&pb, hb, cudaIpcMemLazyEnablePeerAccess);
+    if (e != cudaSuccess) return sticky(h, e);
+    h->opened[h->n_opened++] = pb;
+    blks[q] = static_cast<unsigned char*>(pb);
+    if (q == prev || q == next) {
+      cudaIpcMemHandle_t hm;
+      unsigned long long off;
+      std::memcpy(&hm, b, sizeof(hm));
+      std::memcpy(&off, b + 64, sizeof(off));
+      void* pm = nullptr;
+      e = cudaIpcOpenMemHandle(&pm, hm, cudaIpcMemLazyEnablePeerAccess);
+      if (e != cudaSuccess) return sticky(h, e);
+      h->opened[h->n_opened++] = pm;
+      mbs[q] = reinterpret_cast<float*>(static_cast<unsigned char*>(pm) + off);
+    }
+  }
+  set_peers(h, mbs[prev], mbs[next], blks);
+  return PF_OK;
+}
+
+pf_status pf_peer_connect_local(pf_handle* const* handles, int32_t world) {
+  if (!handles || world < 2 || world > pf::kMaxRanks) return PF_EINVAL;
+  unsigned char* blks[pf::kMaxRanks] = {};
+  for (int q = 0; q < world; ++q) {
+    pf_handle* h = handles[q];
+    pf_status st = peer_check(h);
+    if (st != PF_OK) return st;
+    if (h->cfg.world != world || h->cfg.rank != q) return PF_EINVAL;
+    if ((st = ensure_block(h)) != PF_OK) return st;
+    blks[q] = h->own_blk;
+  }
+  for (int q = 0; q < world; ++q) {
+    pf_handle* h = handles[q];
+    set_peers(h, handles[(q + world - 1) % world]->mailbox, handles[(q + 1) % world]->mailbox, blks);
+  }
+  return PF_OK;
+}
+
+int32_t pf_peer_connected(const pf_handle* h) { return h && h->peers ? 1 : 0; }
+
 pf_status pf_destroy(pf_handle* h) {
   if (!h) return PF_OK;
   cudaStreamSynchronize(h->stream);
+  for (int i = 0; i < h->n_opened; ++i) cudaIpcCloseMemHandle(h->opened[i]);
+  if (h->own_blk) cudaFree(h->own_blk);
   if (h->rec_host) cudaFreeHost(h->rec_host);
   if (h->d_src) cudaFree(h->d_src);
   if (h->d_anc) cudaFree(h->d_anc);

@@ -18,6 +18,7 @@ and the pf_shard comment in include/pf.h.
 """
 from __future__ import annotations
 
+import os
 from dataclasses import dataclass
 
 import torch
@@ -121,23 +122,53 @@ def loopback_exchange(mailboxes: list[torch.Tensor], plan: list[Transfer]) -> No
         mailboxes[t.dst][t.dst_row:t.dst_row + t.nrows].copy_(mailboxes[t.src][t.src_row:t.src_row + t.nrows])
 
 
+def connect_peers(pf, group=None) -> bool:
+    """Peer transport (include/pf.h): every rank exports its CUDA IPC blob, the
+    blobs are all-gathered (host objects, any backend), every rank opens its
+    neighbours' mailboxes and all peer blocks.  Returns False on every rank
+    (nothing connected: the NCCL path stays) if any rank cannot export."""
+    try:
+        blob, ok = pf.peer_export(), True
+    except Exception:   # e.g. no CUDA IPC on this system
+        blob, ok = b"", False
+    got = [None] * pf.world
+    dist.all_gather_object(got, (ok, blob), group=group)
+    if not all(g[0] for g in got):
+        return False
+    pf.peer_connect(b"".join(g[1] for g in got))
+    dist.barrier(group=group)   # every rank connected before anyone steps
+    return True
+
+
 class DistributedFilter:
     """One rank of a filter sharded over ``world`` processes (one per GPU).
 
-    step(): halo exchange of the previous step's mailbox, the step kernel,
-    then all-gather of the per-rank estimate records and their exact reduce,
-    all on the filter's CUDA stream.
+    transport "p2p" (default for ring / torus): the step kernel itself writes
+    the boundary rows into the neighbours' halo rows and reduces the global
+    estimate through the ranks' peer blocks (NVLink peer memory, include/pf.h
+    pf_peer_*), so step() is the kernel launch alone.  transport "nccl" (and
+    All-to-All): halo exchange of the previous step's mailbox through
+    torch.distributed, the step kernel, then all-gather of the per-rank
+    estimate records and their exact reduce, all on the filter's CUDA stream.
     """
 
-    def __init__(self, pf, group=None):
+    def __init__(self, pf, group=None, transport: str | None = None):
         self.pf, self.group = pf, group
         self.rank, self.world = pf.rank, pf.world
         s = pf.shard
         self.plan = halo_plan(pf.topo, pf.n_filters, pf.world, int(s.torus_rows), int(s.torus_cols))
         self.k = 0
         self._records = torch.empty(self.world, s.record_floats, dtype=torch.float32, device=pf.device)
+        transport = transport or os.environ.get("PF_TRANSPORT", "p2p")
+        self.p2p = False
+        if self.world > 1 and transport == "p2p" and pf.topo in (RING, TORUS):
+            self.p2p = connect_peers(pf, group)
 
     def step(self, z, u) -> None:
+        if self.p2p:   # halo + global estimate inside the kernel
+            self.pf.step(z, u)
+            self.k += 1
+            return
         if self.world > 1 and self.k >= 1:
             exchange_halos(self.pf.mailbox[self.k & 1], self.plan, self.rank, self.group)
         self.pf.step(z, u)

@@ -153,6 +153,24 @@ class ParticleFilter:
         B.pf_step_batch(self.h, zs.shape[0], zs.data_ptr(), us.data_ptr(), None if est is None else est.data_ptr())
         self._k += zs.shape[0]
 
+    # -- peer transport (include/pf.h: halo + global estimate inside the step
+    #    kernel over NVLink peer memory) ------------------------------------
+    def peer_export(self) -> bytes:
+        return B.pf_peer_export(self.h)
+
+    def peer_connect(self, blobs: bytes) -> None:
+        B.pf_peer_connect(self.h, blobs)
+
+    @staticmethod
+    def peer_connect_local(filters) -> None:
+        """Connect the shards of ONE process (tests on one device; each shard
+        must step on its own stream)."""
+        B.pf_peer_connect_local([f.h for f in filters])
+
+    @property
+    def peer_connected(self) -> bool:
+        return B.pf_peer_connected(self.h)
+
     def estimate(self):
         """(x_hat [d], logw, global index) of the particle with the highest weight."""
         st = self._est_fn(self.h, self._xhat_p, self._lw_ref, self._idx_ref)
