@@ -160,9 +160,17 @@ def run_ours(a) -> None:
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    # one rank per GPU over NCCL; with fewer visible GPUs than ranks (a
+    # functional check of the multi-rank path on one device) ranks share GPUs
+    # and the host-side plumbing runs over gloo
+    shared = world > 1 and torch.cuda.device_count() < world
+    local = local % torch.cuda.device_count()
     torch.cuda.set_device(local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if shared:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     dev = torch.device("cuda", local)
     K, Wm = a.steps, max(a.warmup, 3)
     T = Wm + K + 8
@@ -181,7 +189,7 @@ def run_ours(a) -> None:
     def max_over_ranks(x: float) -> float:
         if world == 1:
             return x
-        t = torch.tensor([x], dtype=torch.float64, device=dev)
+        t = torch.tensor([x], dtype=torch.float64, device="cpu" if shared else dev)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         return float(t.item())
 
@@ -309,6 +317,8 @@ def run_ours(a) -> None:
                     "ms_per_step": e2e_ms, "h2d_bytes_per_step": 4 * (NJ + 2 + NJ),
                     "d2h_bytes_per_step": 4 * (4 + D)},
             "clocks": clocks, "gpu_launches": K * (1 if (world == 1 or transport["p2p"]) else 2), **extras}
+    if shared:
+        line["config"]["shared_gpus"] = "functional check: ranks share GPUs (gloo host plumbing); not a timing"
     if world > 1:
         line["config"]["transport"] = ("nvlink peer stores + device rendezvous in the step kernel" if transport["p2p"]
                                        else "nccl send/recv halos + all-gather of records")
