@@ -1404,12 +1404,14 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
   const unsigned long long tl_epi = tl_now();
 #endif
   __shared__ unsigned int s_last;
+  // peer transport: every thread that stored into a neighbour's halo orders
+  // those NVLink stores itself (system scope) before the CTA's completion count
+  if (P.peer_mb[0]) __threadfence_system();
   __syncthreads();
   if (threadIdx.x == 0) {
     // the CTA barrier orders every thread's writes (mailbox rows, key) before
     // thread 0's cumulative gpu-scope fence and the completion count
-    if (P.peer_mb[0]) __threadfence_system();   // this CTA's peer halo stores before the count
-    else __threadfence();
+    __threadfence();
     const unsigned int prev = atomicAdd(P.counter, 1u);
     s_last = (prev == gridDim.x - 1) ? 1u : 0u;
   }
