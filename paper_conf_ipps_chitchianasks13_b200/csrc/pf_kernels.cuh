@@ -720,26 +720,28 @@ struct SampleChunked2 {
 // distributed.py): ring — local sub-filter 0 -> the previous rank's row
 // n_local + 1, the last -> the next rank's row n_local; torus — the first grid
 // row -> the rank above, rows n_local + C + c, the last grid row -> the rank
-// below, rows n_local + c.  The row's first t entries [logw, index bits, x],
-// copied by one warp (out of line: no register cost in the step loop).
+// below, rows n_local + c.  The rows' first t entries [logw, index bits, x],
+// copied by the last CTA (every row is complete; no code in the step loop).
 template <int E>
-__device__ __noinline__ void peer_halo_copy(const StepParams& P, long long n, int lane) {
+__device__ void peer_halo_rows(const StepParams& P) {   // whole CTA (the last one)
   const long long nl = P.n_local, par = static_cast<long long>(P.k & 1u) * P.mb_parity;
-  long long row0 = -1, row1 = -1;   // destination rows in the previous / next rank
-  if (P.topo == TOPO_RING) {
-    if (n == 0) row0 = nl + 1;
-    if (n == nl - 1) row1 = nl;
-  } else {
-    const long long Cc = P.C, lr = n / Cc, c = n - lr * Cc, rows = nl / Cc;
-    if (lr == 0) row0 = nl + Cc + c;
-    if (lr == rows - 1) row1 = nl + c;
-  }
-  if (row0 < 0 && row1 < 0) return;
-  const float* src = P.mb_cur + n * P.tt * E;   // the row's first t entries
-  for (int e = lane; e < P.t * E; e += 32) {
-    const float v = __ldcg(src + e);
-    if (row0 >= 0) P.peer_mb[0][par + row0 * P.tt * E + e] = v;
-    if (row1 >= 0) P.peer_mb[1][par + row1 * P.tt * E + e] = v;
+  const int per = P.t * E;                                  // the row's first t entries
+  const long long Cc = P.topo == TOPO_RING ? 1 : P.C;       // rows per side
+  const long long total = 2 * Cc * per;
+  for (long long i = threadIdx.x; i < total; i += blockDim.x) {
+    const int side = static_cast<int>(i / (Cc * per));      // 0: -> previous rank, 1: -> next rank
+    const long long j = i - side * Cc * per;
+    const long long c = j / per;
+    const int e = static_cast<int>(j - c * per);
+    long long src, dst;
+    if (P.topo == TOPO_RING) {
+      src = side == 0 ? 0 : nl - 1;
+      dst = side == 0 ? nl + 1 : nl;
+    } else {
+      src = side == 0 ? c : nl - Cc + c;
+      dst = side == 0 ? nl + Cc + c : nl + c;
+    }
+    P.peer_mb[side][par + dst * P.tt * E + e] = __ldcg(P.mb_cur + src * P.tt * E + e);
   }
 }
 
@@ -1379,10 +1381,6 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
       }
     }
     finish();
-    // peer transport: a boundary sub-filter's best-t row (complete in this
-    // rank's mailbox after finish()'s group barrier) also goes straight into
-    // the neighbour rank's halo row (NVLink stores)
-    if (P.peer_mb[0] && (mode == MODE_STEP || mode == MODE_PUBLISH) && G.wig == 0) peer_halo_copy<E>(P, n, G.lane);
 #ifdef PF_TIMELINE
     if (G.t == 0) {
       const unsigned long long tl_end = tl_now();
@@ -1404,9 +1402,6 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
   const unsigned long long tl_epi = tl_now();
 #endif
   __shared__ unsigned int s_last;
-  // peer transport: every thread that stored into a neighbour's halo orders
-  // those NVLink stores itself (system scope) before the CTA's completion count
-  if (P.peer_mb[0]) __threadfence_system();
   __syncthreads();
   if (threadIdx.x == 0) {
     // the CTA barrier orders every thread's writes (mailbox rows, key) before
@@ -1426,10 +1421,12 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
       const float* blk = P.parts + (col / M) * C::ROW + (col % M);
       float* outs[3] = {P.record, P.est_out, P.record_host};
       if (P.peer_mb[0] && (mode == MODE_STEP || mode == MODE_PUBLISH)) {
-        // peer transport: this shard's best record into slot `rank` of every
-        // rank's peer block, then step flags, then wait for every rank's flag
+        // peer transport: the boundary sub-filters' best-t rows into the
+        // neighbour ranks' halo rows, this shard's best record into slot
+        // `rank` of every rank's peer block, then step flags, then wait for every rank's flag
         // (device-side rendezvous over NVLink), then the exact max over the
         // world records (the all-gather + pf_reduce_records of the NCCL path)
+        peer_halo_rows<E>(P);
         if (tid < D) {
           const float v = __ldcg(blk + tid * M);
           for (int r = 0; r < P.world; ++r) peer_rec(P.peer_blk[r], P.rank)[4 + tid] = v;
