@@ -30,6 +30,7 @@ for key, lab in (("C5_nj5_16M", "16M particles d = 9 (RWS)"), ("C4_nj28_16M_rws"
              f"{v['lane_instr_per_particle']:.0f} lane-instr/particle, issue active {v['smsp__issue_active.avg.pct_of_peak_sustained_active']:.0f} % |")
 L.append(f"| 10⁸ particles (d = 9, sweep) | {e8['us_per_step']:.0f} µs/step = {e8['hbm_gbs_algorithmic']:.0f} GB/s ({100*e8['hbm_gbs_algorithmic']/peak:.0f} %) |")
 L.append(f"| CPU oracle (plain C, 1 core) | {b['cpu_baseline']['value']:.3g} particle-steps/s ({b['cpu_baseline']['sample']}); reference arm {ref['value']:.3g} |")
+L.append("| 2 ranks sharing one GPU (peer transport, functional check; `profiles/r01_bench_2rank_shared_gpu.json`) | completes; time-sliced on one device, not a scaling number |")
 L.append("| Paper (GTX 580/680, HD 7970; Table III) | \"a few hundred\" estimates/s at 1M (context only) |\n")
 L.append("Sweeps (`scripts/sweeps.py`, device-resident inputs, L2 flushed per step):\n")
 L.append("| Sweep | d | m | N | particles | resampler | X, t | policy | µs/step | particle-steps/s | alg. HBM GB/s |")
