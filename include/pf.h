@@ -305,7 +305,10 @@ pf_status pf_debug_check_sqrt(uint32_t lo_bits, uint32_t hi_bits, uint64_t* mism
  *    raises its step flag there (system-scope release) and waits for every
  *    rank's flag (acquire): a device-side rendezvous per step, after which the
  *    exact max over the world records is the global estimate on every rank.
- * Ring and 2D torus, world 2..8, steps strictly increasing after connecting.
+ * All-to-All: the shard's pool row (its best t) goes into every rank's peer
+ * block and the global pool is reduced after the rendezvous (pf_reduce_pool,
+ * fused).  Ring, 2D torus, All-to-All; world 2..8; steps strictly increasing
+ * after connecting.
  * pf_peer_export: this rank's blob (CUDA IPC handles of the caller's mailbox
  *   allocation + offset, and of a 4 KiB runtime-owned peer block; the rank).
  *   Host blob[PF_PEER_BLOB_BYTES].  Call before the first step.
@@ -315,8 +318,7 @@ pf_status pf_debug_check_sqrt(uint32_t lo_bits, uint32_t hi_bits, uint64_t* mism
  * pf_peer_connect_local: the same for `world` handles of ONE process (tests on
  *   one device; their steps must run on different streams).
  * Errors: PF_ESTATE (world == 1, central filter, already stepped / connected,
- *   export missing), PF_EUNSUPPORTED (All-to-All: its pool keeps the NCCL path),
- *   PF_ECUDA (IPC failure; the handle stays on the NCCL path). */
+ *   export missing), PF_ECUDA (IPC failure; the handle stays on the NCCL path). */
 #define PF_PEER_BLOB_BYTES 160
 pf_status pf_peer_export(pf_handle* h, uint8_t* blob);
 pf_status pf_peer_connect(pf_handle* h, const uint8_t* blobs);

@@ -53,6 +53,7 @@ constexpr int kRecordSeq = 127;
 // [kMaxRanks] u64 step flags, then [kMaxRanks][kPeerRec] float records.
 constexpr int kMaxRanks = 8;
 constexpr int kPeerRec = 40;   // 4 + d <= 36 floats, padded
+constexpr int kPeerPool = 32 * 34;   // All-to-All: t <= 32 entries of E = d + 2 <= 34 floats
 
 struct StepParams {
   ArmConsts mc;
@@ -751,6 +752,9 @@ __device__ __forceinline__ unsigned long long* peer_flags(unsigned char* blk) {
 __device__ __forceinline__ float* peer_rec(unsigned char* blk, int r) {
   return reinterpret_cast<float*>(blk + sizeof(unsigned long long) * kMaxRanks) + r * kPeerRec;
 }
+__device__ __forceinline__ float* peer_pool(unsigned char* blk, int r) {
+  return peer_rec(blk, kMaxRanks) + r * kPeerPool;
+}
 
 // Best t of the union of two descending lists held by lanes 0..t-1 (run list
 // r, new list nb; keys unique or 0 = empty) into r, by t rounds of warp max.
@@ -1414,6 +1418,27 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
   if (s_last) {
     __threadfence();
     const int tid = threadIdx.x;
+    // All-to-All: this shard's best t -> pool row pool_local_row (first: the
+    // peer transport also ships it to every rank before the rendezvous)
+    if (P.topo == TOPO_A2A && P.t > 0 && mode != MODE_EXCHANGE) {
+      float* pool = P.mb_cur + P.pool_local_row * P.tt * E;
+      if (P.t == 1) {   // the pool's best is the shard's best particle: the record just written
+        const u64 key = __ldcg(P.key_cur);
+        const uint32_t gidx = 0xFFFFFFFFu - static_cast<uint32_t>(key);
+        const long long col = static_cast<long long>(gidx) - P.g0 * M;
+        const float* blk = P.parts + (col / M) * C::ROW + (col % M);
+        if (tid < D) pool[2 + tid] = __ldcg(blk + tid * M);
+        if (tid == 0) {
+          pool[0] = unord_f32(static_cast<uint32_t>(key >> 32));
+          pool[1] = __uint_as_float(gidx);
+        }
+      } else {
+        // reduction scratch: group 0's stage buffer (no load in flight after the loop)
+        u64* red = reinterpret_cast<u64*>(smem + C::c_groups + C::g_stage);
+        if (P.pool_cta) pool_top_t_cta<E>(P, pool, red, static_cast<long long>(gridDim.x) * C::S);
+        else pool_top_t<E>(P, P.mb_cur, P.n_local * P.t, pool, red);
+      }
+    }
     if (mode != MODE_EXCHANGE) {
       const u64 key = __ldcg(P.key_cur);
       const uint32_t gidx = 0xFFFFFFFFu - static_cast<uint32_t>(key);
@@ -1426,7 +1451,17 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
         // `rank` of every rank's peer block, then step flags, then wait for every rank's flag
         // (device-side rendezvous over NVLink), then the exact max over the
         // world records (the all-gather + pf_reduce_records of the NCCL path)
-        peer_halo_rows<E>(P);
+        const bool a2a = P.topo == TOPO_A2A && P.t > 0;
+        if (a2a) {
+          __syncthreads();   // the local pool row is complete
+          const float* lp = P.mb_cur + P.pool_local_row * P.tt * E;
+          for (int i = tid; i < P.world * P.t * E; i += blockDim.x) {
+            const int r = i / (P.t * E), e = i - r * (P.t * E);
+            peer_pool(P.peer_blk[r], P.rank)[e] = __ldcg(lp + e);
+          }
+        } else {
+          peer_halo_rows<E>(P);
+        }
         if (tid < D) {
           const float v = __ldcg(blk + tid * M);
           for (int r = 0; r < P.world; ++r) peer_rec(P.peer_blk[r], P.rank)[4 + tid] = v;
@@ -1464,6 +1499,32 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
             for (int o = 0; o < 3; ++o)
               if (outs[o]) outs[o][c] = v;
           }
+          if (a2a) {   // the global pool: best t of the world's pool rows (pf_reduce_pool, fused)
+            float* out = P.mb_cur + P.pool_row * P.tt * E;
+            u64 prev = ~0ull;
+            for (int jb = 0; jb < P.t; ++jb) {
+              u64 best = 0ull;
+              int be = -1;
+              for (int e = tid; e < P.world * P.t; e += 32) {
+                const int r = e / P.t, jj = e - r * P.t;
+                const float* en = peer_pool(P.peer_blk[P.rank], r) + jj * E;
+                const u64 kk2 = order_key(__ldcv(en), __float_as_uint(__ldcv(en + 1)));
+                if (kk2 < prev && kk2 > best) {
+                  best = kk2;
+                  be = e;
+                }
+              }
+              const u64 g2 = warp_max_u64(best);
+              const int own = __ffs(__ballot_sync(0xFFFFFFFFu, be >= 0 && best == g2)) - 1;
+              const int bsel = __shfl_sync(0xFFFFFFFFu, be, own < 0 ? 0 : own);
+              if (own >= 0) {
+                const int r = bsel / P.t, jj = bsel - r * P.t;
+                const float* en = peer_pool(P.peer_blk[P.rank], r) + jj * E;
+                for (int c = tid; c < E; c += 32) out[jb * E + c] = __ldcv(en + c);
+              }
+              prev = g2;
+            }
+          }
         }
       } else {
         if (tid < D) {
@@ -1486,25 +1547,6 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
         __threadfence_system();
         __syncthreads();
         if (tid == 0) *reinterpret_cast<volatile uint32_t*>(P.record_host + kRecordSeq) = P.k;
-      }
-    }
-    if (P.topo == TOPO_A2A && P.t > 0 && mode != MODE_EXCHANGE) {
-      float* pool = P.mb_cur + P.pool_local_row * P.tt * E;
-      if (P.t == 1) {   // the pool's best is the shard's best particle: the record just written
-        const u64 key = __ldcg(P.key_cur);
-        const uint32_t gidx = 0xFFFFFFFFu - static_cast<uint32_t>(key);
-        const long long col = static_cast<long long>(gidx) - P.g0 * M;
-        const float* blk = P.parts + (col / M) * C::ROW + (col % M);
-        if (tid < D) pool[2 + tid] = __ldcg(blk + tid * M);
-        if (tid == 0) {
-          pool[0] = unord_f32(static_cast<uint32_t>(key >> 32));
-          pool[1] = __uint_as_float(gidx);
-        }
-      } else {
-        // reduction scratch: group 0's stage buffer (no load in flight after the loop)
-        u64* red = reinterpret_cast<u64*>(smem + C::c_groups + C::g_stage);
-        if (P.pool_cta) pool_top_t_cta<E>(P, pool, red, static_cast<long long>(gridDim.x) * C::S);
-        else pool_top_t<E>(P, P.mb_cur, P.n_local * P.t, pool, red);
       }
     }
     if (tid == 0) {

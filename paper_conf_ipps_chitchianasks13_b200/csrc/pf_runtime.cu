@@ -964,14 +964,17 @@ pf_status pf_get_trace(pf_handle* h, int64_t* src, int32_t* ancestors) {
 
 // ---- peer transport (NVLink / NVSwitch peer memory via CUDA IPC) ----------
 namespace {
-constexpr size_t kPeerBlockBytes = 4096;   // [kMaxRanks] u64 flags + [kMaxRanks][kPeerRec] floats
-static_assert(sizeof(u64) * pf::kMaxRanks + sizeof(float) * pf::kMaxRanks * pf::kPeerRec <= kPeerBlockBytes, "");
+// [kMaxRanks] u64 flags + [kMaxRanks][kPeerRec] record floats + [kMaxRanks][kPeerPool] pool floats
+constexpr size_t kPeerBlockBytes = 40960;
+static_assert(sizeof(u64) * pf::kMaxRanks + sizeof(float) * pf::kMaxRanks * (pf::kPeerRec + pf::kPeerPool) <=
+                  kPeerBlockBytes, "");
 
 pf_status peer_check(const pf_handle* h) {
   if (!h) return PF_EINVAL;
   if (h->err != PF_OK) return h->err;
   if (h->g.central || h->cfg.world < 2 || h->cfg.world > pf::kMaxRanks) return PF_ESTATE;
-  if (h->cfg.topo != PF_TOPO_RING && h->cfg.topo != PF_TOPO_TORUS2D) return PF_EUNSUPPORTED;
+  if (h->cfg.topo != PF_TOPO_RING && h->cfg.topo != PF_TOPO_TORUS2D && h->cfg.topo != PF_TOPO_ALL2ALL)
+    return PF_EUNSUPPORTED;
   if (h->step != 0 || h->peers) return PF_ESTATE;   // connect once, before the first step
   return PF_OK;
 }

@@ -143,11 +143,11 @@ def connect_peers(pf, group=None) -> bool:
 class DistributedFilter:
     """One rank of a filter sharded over ``world`` processes (one per GPU).
 
-    transport "p2p" (default for ring / torus): the step kernel itself writes
-    the boundary rows into the neighbours' halo rows and reduces the global
-    estimate through the ranks' peer blocks (NVLink peer memory, include/pf.h
-    pf_peer_*), so step() is the kernel launch alone.  transport "nccl" (and
-    All-to-All): halo exchange of the previous step's mailbox through
+    transport "p2p" (default): the step kernel itself writes the boundary rows
+    into the neighbours' halo rows (All-to-All: its pool row into every rank's
+    peer block) and reduces the global estimate (and pool) through the ranks'
+    peer blocks (NVLink peer memory, include/pf.h pf_peer_*), so step() is the
+    kernel launch alone.  transport "nccl": halo exchange of the previous step's mailbox through
     torch.distributed, the step kernel, then all-gather of the per-rank
     estimate records and their exact reduce, all on the filter's CUDA stream.
     """
@@ -161,7 +161,7 @@ class DistributedFilter:
         self._records = torch.empty(self.world, s.record_floats, dtype=torch.float32, device=pf.device)
         transport = transport or os.environ.get("PF_TRANSPORT", "p2p")
         self.p2p = False
-        if self.world > 1 and transport == "p2p" and pf.topo in (RING, TORUS):
+        if self.world > 1 and transport == "p2p":
             self.p2p = connect_peers(pf, group)
 
     def step(self, z, u) -> None:

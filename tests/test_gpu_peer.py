@@ -1,5 +1,5 @@
-"""Peer transport (include/pf.h pf_peer_*): the halo rows and the global
-estimate cross ranks inside the step kernel (peer stores + a device-side flag
+"""Peer transport (include/pf.h pf_peer_*): the halo rows (or the All-to-All
+pool rows) and the global estimate cross ranks inside the step kernel (peer stores + a device-side flag
 rendezvous) instead of NCCL around it.  On one device: (1) `world` shards in
 one process, each stepping on its own stream, connected without IPC; (2) two
 processes sharing the device, connected through CUDA IPC with the blobs
@@ -29,13 +29,14 @@ def P():
 
 
 @pytest.mark.timeout(120)
-@pytest.mark.parametrize("topo,N,world", [("ring", 16, 2), ("ring", 8, 4), ("torus", 64, 2), ("torus", 16, 4),
-                                          ("ring", 4, 4)])
-def test_peer_transport_local(P, orc, W, topo, N, world):
+@pytest.mark.parametrize("topo,N,world,t", [("ring", 16, 2, 1), ("ring", 8, 4, 1), ("torus", 64, 2, 1),
+                                            ("torus", 16, 4, 1), ("ring", 4, 4, 1), ("all2all", 16, 2, 2),
+                                            ("all2all", 8, 4, 1), ("all2all", 32, 4, 3)])
+def test_peer_transport_local(P, orc, W, topo, N, world, t):
     import torch
     nj, m, T = 5, 64, 6
     tr = W.make_trajectory(nj, T, 5)
-    kw = dict(m=m, n_filters=N, t=1, topo=topo, resampler="rws", seed=31)
+    kw = dict(m=m, n_filters=N, t=t, topo=topo, resampler="rws", seed=31)
     shards = [P.ParticleFilter(tr["mu0"], tr["sigma0"], P.ArmModel(n_joints=nj), rank=r, world=world,
                                stream=torch.cuda.Stream(), **kw) for r in range(world)]
     P.ParticleFilter.peer_connect_local(shards)
@@ -69,7 +70,7 @@ _TWO_PROC = textwrap.dedent(r"""
     torch.cuda.set_device(0)
     nj, m, N, T, topo = 5, 64, 16, 5, os.environ["PF_TOPO"]
     tr = W.make_trajectory(nj, T, 6)
-    kw = dict(m=m, n_filters=N, t=1, topo=topo, resampler="vose", seed=13)
+    kw = dict(m=m, n_filters=N, t=2 if topo == "all2all" else 1, topo=topo, resampler="vose", seed=13)
     pf = F.ParticleFilter(tr["mu0"], tr["sigma0"], F.ArmModel(n_joints=nj), rank=rank, world=world, **kw)
     df = D.DistributedFilter(pf, transport="p2p")
     assert df.p2p and pf.peer_connected
@@ -91,7 +92,7 @@ _TWO_PROC = textwrap.dedent(r"""
 
 
 @pytest.mark.timeout(300)
-@pytest.mark.parametrize("topo", ["ring", "torus"])
+@pytest.mark.parametrize("topo", ["ring", "torus", "all2all"])
 def test_peer_transport_two_processes_ipc(P, topo, tmp_path):
     root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
     script = tmp_path / "peer2.py"
