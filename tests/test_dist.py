@@ -166,3 +166,47 @@ def test_mean_protocol_gloo(world):
     ret = ctx.Manager().dict()
     mp.start_processes(_mean_worker, args=(world, _free_port(), ret), nprocs=world, join=True, start_method="spawn")
     assert len(ret) == world
+
+
+class _FakePeerShard:
+    """Host stand-in for the peer-transport handshake of a shard: export may
+    fail (no CUDA IPC), connect records the blobs it was given."""
+
+    def __init__(self, rank, world, can_export):
+        self.rank, self.world, self.can_export, self.connected = rank, world, can_export, None
+
+    def peer_export(self):
+        if not self.can_export:
+            raise RuntimeError("no CUDA IPC")
+        return bytes([self.rank]) * 160
+
+    def peer_connect(self, blobs):
+        self.connected = blobs
+
+
+def _peer_worker(rank, world, port, fail_rank, ret):
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        pf = _FakePeerShard(rank, world, rank != fail_rank)
+        ok = Dd.connect_peers(pf)
+        ret[rank] = (ok, pf.connected)
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world,fail_rank", [(2, -1), (3, -1), (2, 1), (3, 0)])
+def test_peer_handshake_gloo(world, fail_rank):
+    # every rank connects with all blobs in rank order, or (one rank cannot
+    # export) no rank connects and all stay on the NCCL transport
+    ctx = mp.get_context("spawn")
+    ret = ctx.Manager().dict()
+    mp.start_processes(_peer_worker, args=(world, _free_port(), fail_rank, ret), nprocs=world, join=True,
+                       start_method="spawn")
+    expect = b"".join(bytes([r]) * 160 for r in range(world))
+    for r in range(world):
+        ok, blobs = ret[r]
+        if fail_rank < 0:
+            assert ok and blobs == expect
+        else:
+            assert not ok and blobs is None
