@@ -688,8 +688,10 @@ pf_status pf_estimate(pf_handle* h, float* x_hat, float* logw, int64_t* idx) {
         if (e != cudaErrorNotReady) break;
       }
     }
-    if (e == cudaSuccess || e == cudaErrorNotReady) e = cudaStreamQuery(h->stream);
-    if (e == cudaErrorNotReady) e = cudaSuccess;   // the record is complete; the kernel is retiring
+    // the step number arrived after the record (system-scope fence): the
+    // record is complete.  A device error ends the poll through the query
+    // above; one raised after the record surfaces at the next call (sticky).
+    if (e == cudaErrorNotReady) e = cudaSuccess;
     if (e != cudaSuccess) return sticky(h, e);
   } else {
     e = cudaMemcpyAsync(h->rec_host, record(h), sizeof(float) * (4 + h->g.d), cudaMemcpyDeviceToHost, h->stream);
