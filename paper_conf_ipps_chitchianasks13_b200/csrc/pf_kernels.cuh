@@ -934,6 +934,12 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
     mbar_init(bars, 1);
     mbar_init(bars + 1, 1);
     fence_mbar_init();
+  }
+  // programmatic dependent launch: everything above overlaps the previous
+  // step's tail; nothing it wrote (particle blocks, mailbox, counters, key,
+  // device inputs) is read before its grid has completed (no-op otherwise)
+  asm volatile("griddepcontrol.wait;" ::: "memory");
+  if (G.t == 0) {
     issue(0, gid0);
     if (gid0 < P.n_local) pending = atomicAdd(P.work, 1u);
   }
@@ -1401,6 +1407,10 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
 #endif
   }
 
+  // this CTA's sub-filters are done: the next step's grid may start launching
+  // into the SMs the retiring CTAs free (it waits in griddepcontrol.wait)
+  asm volatile("griddepcontrol.launch_dependents;");
+
   // ---- a5: the last CTA to finish copies the winning particle (R6)
 #ifdef PF_TIMELINE
   const unsigned long long tl_epi = tl_now();
@@ -1614,9 +1624,24 @@ struct StepKernel {
     if (e != cudaSuccess) return e;
     return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, pf_step_kernel<C>, C::T * C::S, smem());
   }
-  static cudaError_t launch(const StepParams& p, int grid, cudaStream_t s) {
-    pf_step_kernel<C><<<grid, C::T * C::S, smem(), s>>>(p);
-    return cudaGetLastError();
+  static cudaError_t launch(const StepParams& p, int grid, cudaStream_t s, bool pdl) {
+    // programmatic stream serialization: back-to-back steps overlap the launch
+    // and prologue of step k + 1 with the tail of step k (see the kernel)
+    if (!pdl) {
+      pf_step_kernel<C><<<grid, C::T * C::S, smem(), s>>>(p);
+      return cudaGetLastError();
+    }
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(grid);
+    cfg.blockDim = dim3(C::T * C::S);
+    cfg.dynamicSmemBytes = smem();
+    cfg.stream = s;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    return cudaLaunchKernelEx(&cfg, pf_step_kernel<C>, p);
   }
   static cudaError_t resample_debug(const uint32_t* q, const uint32_t* ua, const uint32_t* ub, int* anc, u64* prob,
                                     int* alias, long long N, cudaStream_t s) {

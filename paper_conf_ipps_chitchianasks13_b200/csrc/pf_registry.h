@@ -19,7 +19,7 @@ struct KernelEntry {
   int gw, s, nstage, unr, minb;   // warps per group, groups per CTA, TMA stages, sample unroll, min CTAs/SM
   int large;                      // preferred when the shard has >= kLargeNLocal sub-filters
   cudaError_t (*prepare)(int* blocks_per_sm);
-  cudaError_t (*launch)(const StepParams& p, int grid, cudaStream_t s);
+  cudaError_t (*launch)(const StepParams& p, int grid, cudaStream_t s, bool pdl);
   cudaError_t (*resample_debug)(const uint32_t* q, const uint32_t* ua, const uint32_t* ub, int* anc,
                                 unsigned long long* prob, int* alias, long long N, cudaStream_t s);
   size_t smem;

@@ -201,6 +201,8 @@ struct pf_handle {
   // peer transport (pf_peer_connect*): the neighbour ranks' mailboxes and every
   // rank's peer block (flags + records), this rank's own block (cudaMalloc'd)
   bool peers;
+  bool local_peers;   // connected by pf_peer_connect_local (one process, one device)
+  bool pdl;           // programmatic dependent launch of the step kernel (PF_NO_PDL unset at init)
   float* peer_mb[2];
   unsigned char* peer_blk[pf::kMaxRanks];
   unsigned char* own_blk;
@@ -368,7 +370,10 @@ pf::CentralParams central_params(pf_handle* h, long long k) {
 }
 
 pf_status launch(pf_handle* h, const pf::StepParams& p) {
-  return sticky(h, h->ke->launch(p, h->grid, h->stream));
+  // programmatic dependent launch, except for shards of one process sharing a
+  // device through the peer transport (a next step's waiting CTAs could hold
+  // the SMs another shard's current step needs to reach the rendezvous)
+  return sticky(h, h->ke->launch(p, h->grid, h->stream, h->pdl && !h->local_peers));
 }
 pf_status launch_central(pf_handle* h, const pf::CentralParams& c) {
   return sticky(h, pf::central_step(h->g.nj, c, h->grid, h->stream));
@@ -532,6 +537,7 @@ pf_status pf_init(const pf_config* cfg, const pf_model_params* model, const pf_b
   if (e == cudaSuccess) e = cudaHostGetDevicePointer(reinterpret_cast<void**>(&h->rec_host_dev), h->rec_host, 0);
   if (e == cudaSuccess) {
     h->mapped = std::getenv("PF_NO_MAPPED") == nullptr;
+    h->pdl = std::getenv("PF_NO_PDL") == nullptr;
     h->last_mapped = false;
     reinterpret_cast<volatile uint32_t*>(h->rec_host)[pf::kRecordSeq] = 0xFFFFFFFFu;
   }
@@ -1082,6 +1088,7 @@ pf_status pf_peer_connect_local(pf_handle* const* handles, int32_t world) {
   for (int q = 0; q < world; ++q) {
     pf_handle* h = handles[q];
     set_peers(h, handles[(q + world - 1) % world]->mailbox, handles[(q + 1) % world]->mailbox, blks);
+    h->local_peers = true;
   }
   return PF_OK;
 }
