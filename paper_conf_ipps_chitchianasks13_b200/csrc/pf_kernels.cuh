@@ -930,16 +930,14 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
     return nn;
   };
 
+  // programmatic dependent launch: the CTA's launch overlaps the previous
+  // step's tail; nothing that step wrote (particle blocks, mailbox, counters,
+  // key, device inputs) is read before its grid has completed (no-op otherwise)
+  asm volatile("griddepcontrol.wait;" ::: "memory");
   if (G.t == 0) {
     mbar_init(bars, 1);
     mbar_init(bars + 1, 1);
     fence_mbar_init();
-  }
-  // programmatic dependent launch: everything above overlaps the previous
-  // step's tail; nothing it wrote (particle blocks, mailbox, counters, key,
-  // device inputs) is read before its grid has completed (no-op otherwise)
-  asm volatile("griddepcontrol.wait;" ::: "memory");
-  if (G.t == 0) {
     issue(0, gid0);
     if (gid0 < P.n_local) pending = atomicAdd(P.work, 1u);
   }
