@@ -426,7 +426,15 @@ __device__ __forceinline__ void resample_group(const uint32_t (&q)[C::P], const 
     // per-slot class, deficit, counts and E are recomputed from them.
     u64 qinc[P], pinc[P];
     u64 Qg, ptot;
-    {
+    if constexpr (C::SCAN32) {   // Q <= M 2^22 fits 32 bits: the weight scan in u32
+      uint32_t val[P];
+#pragma unroll
+      for (int j = 0; j < P; ++j) val[j] = q[j];
+      uint32_t* b32 = reinterpret_cast<uint32_t*>(S.scan);
+      Qg = slot_scan_smem<C, uint32_t>(val, b32, G);
+#pragma unroll
+      for (int j = 0; j < P; ++j) qinc[j] = b32[C::slot(G.t, j)];
+    } else {
       u64 val[P];
 #pragma unroll
       for (int j = 0; j < P; ++j) val[j] = q[j];
