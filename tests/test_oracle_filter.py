@@ -151,3 +151,23 @@ def test_central_slots_equals_whole_filter(orc, W):
         os_, ow = orc.central_slots(cfg, md, s0, w0, 3, tr["Z"][3], tr["U"][2], slots)
         np.testing.assert_array_equal(os_, s1[:, slots])
         np.testing.assert_array_equal(ow, w1[slots])
+
+
+@pytest.mark.parametrize("nj,m,N,res", [(2, 64, 16, "rws"), (2, 64, 16, "vose"), (5, 256, 16, "rws")])
+def test_fp32_trajectory_matches_fp64_elementwise(orc, W, nj, m, N, res):
+    # the fp32 contract (F1-F11) against the independent float64 / libm
+    # oracle, element by element over 10 steps (every particle, every step):
+    # within the north_star's 1e-5 relative bar, and no integer decision
+    # (order, exchange, q, ancestor, argmax) differs (§VI)
+    tr = W.make_trajectory(nj, 10, 0)
+    cfg = orc.Config(m=m, n_filters=N, t=1, topo="ring", resampler=res, seed=3)
+    a = orc.Filter(cfg, orc.Model(n_joints=nj), tr["mu0"], tr["sigma0"])
+    b = orc.Filter(cfg, orc.Model(n_joints=nj), tr["mu0"], tr["sigma0"], fp64=True)
+    for k in range(1, 11):
+        a.step(tr["Z"][k], tr["U"][k - 1])
+        b.step(tr["Z"][k], tr["U"][k - 1])
+        s32, w32, _ = a.get()
+        s64, w64, _ = b.get()
+        np.testing.assert_array_less(np.abs(s32 - s64), 1e-5 * np.maximum(1, np.abs(s64)))
+        np.testing.assert_array_less(np.abs(w32 - w64), 1e-5 * np.maximum(1, np.abs(w64)))
+        assert a.estimate()[2] == b.estimate()[2]
