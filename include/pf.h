@@ -43,7 +43,9 @@ typedef enum {
   PF_ENOMEM = -2,        /* host allocation failed                           */
   PF_ECUDA = -3,         /* CUDA error (sticky)                              */
   PF_ESTATE = -5,        /* call not valid in the handle's state             */
-  PF_EUNSUPPORTED = -6   /* (n_joints, m) combination not compiled           */
+  PF_EUNSUPPORTED = -6,  /* (model, n_joints, m) combination not compiled    */
+  PF_ETIMEOUT = -7       /* peer transport: a rank did not reach the device  */
+                         /* rendezvous within PF_PEER_TIMEOUT_MS (sticky)    */
 } pf_status;
 
 /* Exchange scheme X (PAPER.md:18 Table I; :16 Fig.1; :20 §VI-E): Ring and
@@ -54,10 +56,24 @@ typedef enum { PF_TOPO_NONE = 0, PF_TOPO_RING = 1, PF_TOPO_TORUS2D = 2, PF_TOPO_
 /* Resampler (PAPER.md:18 §IV; :20–22 §VI-F). */
 typedef enum { PF_RESAMPLE_RWS = 0, PF_RESAMPLE_VOSE = 1 } pf_resampler;
 /* Model hooks (the paper separates "generic particle filtering from
- * model-specific routines", §I).  The robotic arm of
- * PAPER.md:22–24 §VII-A with h(x) of reading R14; compiled for
- * n_joints in {2, 5, 28}. */
-typedef enum { PF_MODEL_ARM_PLANAR = 0 } pf_model_id;
+ * model-specific routines.  New dynamical system models can be easily
+ * added", §I).  The step kernels are templates over a model
+ * policy (csrc/pf_model.cuh: state / measurement / control dimensions and
+ * the sample (F8) and weight (F10) hooks, fused into the step); a model id
+ * selects the compiled instance.
+ *  PF_MODEL_ARM_PLANAR       the robotic arm of PAPER.md:22–24 §VII-A with
+ *                            h(x) of reading R14; d = n_joints + 4, z has
+ *                            n_joints + 2 entries (x_C, y_C, joint angles),
+ *                            u has n_joints; compiled for n_joints in
+ *                            {2, 5, 28} (others: PF_EUNSUPPORTED).
+ *  PF_MODEL_LINEAR_GAUSS_1D  one joint with its angle sensor and no camera:
+ *                            theta_k = theta_{k-1} + h_s u + w,
+ *                            w ~ N(0, sigma_theta^2); z = theta + v,
+ *                            v ~ N(0, sigma_theta_meas^2); d = 1, z and u
+ *                            one entry each (the Kalman special case of
+ *                            SURVEY §8(c)); n_joints, arm_length,
+ *                            sigma_pos/vel/cam are ignored. */
+typedef enum { PF_MODEL_ARM_PLANAR = 0, PF_MODEL_LINEAR_GAUSS_1D = 1 } pf_model_id;
 
 /* pf_config.flags */
 #define PF_DEVICE_INPUTS 1u   /* pf_step's z / u are device pointers         */
@@ -171,8 +187,9 @@ pf_status pf_init(const pf_config* cfg, const pf_model_params* model, const pf_b
 /* One time step k = (last step) + 1 of Algorithm 2: exchange
  * with the neighbours' best t of step k-1 (l.10–14), normalise + resample
  * locally (l.15–19), sample + weight (l.3–6), local/global estimate (l.8–9).
- * z_k: float[n_joints + 2] = (x_C, y_C, theta_hat_0..), u_{k-1}:
- * float[n_joints].  Host pointers — their values travel to
+ * z_k: float[zd] and u_{k-1}: float[ud], the model's measurement and
+ * control (arm: zd = n_joints + 2 = (x_C, y_C, theta_hat_0..), ud =
+ * n_joints; linear-Gaussian: one each).  Host pointers — their values travel to
  * the device inside the kernel launch, so the buffers may be reused as soon
  * as the call returns — unless PF_DEVICE_INPUTS (device pointers, read by the
  * kernel).  Asynchronous.
@@ -181,8 +198,8 @@ pf_status pf_init(const pf_config* cfg, const pf_model_params* model, const pf_b
  * records (pf_reduce_records) for a global estimate. */
 pf_status pf_step(pf_handle* h, const float* z_k, const float* u_km1);
 
-/* T consecutive steps with device-resident inputs zs [T][n_joints+2] and
- * us [T][n_joints] (device), writing each step's estimate record
+/* T consecutive steps with device-resident inputs zs [T][zd] and
+ * us [T][ud] (device), writing each step's estimate record
  * (4 + d floats, layout of pf_record_ptr) to est [T][4+d] (device, nullable).
  * world == 1 only (PF_ESTATE otherwise).  Asynchronous (T back-to-back
  * launches on the handle's stream, no host synchronization). */
@@ -301,17 +318,24 @@ pf_status pf_debug_check_sqrt(uint32_t lo_bits, uint32_t hi_bits, uint64_t* mism
  *    sub-filter 0 -> rank r-1's row n_local+1, the last -> rank r+1's row
  *    n_local; torus — the first grid row -> rank r-1's rows n_local+C.., the
  *    last -> rank r+1's rows n_local..);
- *  - the last CTA writes the shard's best record into every rank's peer block,
- *    raises its step flag there (system-scope release) and waits for every
- *    rank's flag (acquire): a device-side rendezvous per step, after which the
+ *  - the last CTA writes the shard's best record into every rank's peer block
+ *    (buffer rv & 1 of a double buffer, rv = the rendezvous number: +1 per
+ *    peer-mode launch — pf_step, pf_set_particles — on every rank), raises its
+ *    flag there to rv (system-scope release) and waits for every rank's flag
+ *    to reach rv (acquire): a device-side rendezvous per step, after which the
  *    exact max over the world records is the global estimate on every rank.
+ *    A rank missing for PF_PEER_TIMEOUT_MS (environment, default 30000) ends
+ *    the wait: pf_estimate then returns PF_ETIMEOUT (sticky) instead of the
+ *    device hanging.
  * All-to-All: the shard's pool row (its best t) goes into every rank's peer
  * block and the global pool is reduced after the rendezvous (pf_reduce_pool,
- * fused).  Ring, 2D torus, All-to-All; world 2..8; steps strictly increasing
- * after connecting.
+ * fused).  Ring, 2D torus, All-to-All; world 2..8; every rank calls pf_step /
+ * pf_set_particles in the same sequence.  Peers on the same device (by PCI bus
+ * id) run without programmatic dependent launch.
  * pf_peer_export: this rank's blob (CUDA IPC handles of the caller's mailbox
- *   allocation + offset, and of a 4 KiB runtime-owned peer block; the rank).
- *   Host blob[PF_PEER_BLOB_BYTES].  Call before the first step.
+ *   allocation + offset, and of an 80 KiB runtime-owned peer block; the rank;
+ *   the device's PCI bus id).  Host blob[PF_PEER_BLOB_BYTES].  Call before the
+ *   first step.
  * pf_peer_connect: blobs [world][PF_PEER_BLOB_BYTES] of all ranks in rank order
  *   (e.g. all-gathered through torch.distributed); opens the peers' blocks and
  *   the neighbours' mailboxes (cudaIpcOpenMemHandle, lazy peer access).

@@ -68,8 +68,18 @@ typedef struct {
 int orc_should_resample(int32_t policy, uint64_t param, const uint32_t* q, int32_t m, uint64_t seed, int64_t n,
                         int64_t k);
 
+/* Models ("our application separates generic particle filtering from
+ * model-specific routines", §I):
+ *   ORC_MODEL_ARM_PLANAR       the robotic arm of PAPER.md:22–24 §VII-A (R14)
+ *   ORC_MODEL_LINEAR_GAUSS_1D  one joint with its angle sensor, no camera:
+ *       theta_k = theta_{k-1} + h_s u + w, w ~ N(0, sigma_theta^2),
+ *       z_k = theta_k + v, v ~ N(0, sigma_theta_meas^2)  (d = 1; the Kalman
+ *       special case of SURVEY §8(c), pinned against the Kalman filter) */
+enum { ORC_MODEL_ARM_PLANAR = 0, ORC_MODEL_LINEAR_GAUSS_1D = 1 };
+
 /* Table II model parameters (§VII-A) — fp32 values. */
 typedef struct {
+  int32_t model;           /* ORC_MODEL_*                                   */
   int32_t n_joints;        /* joints incl. base rotation; d = n_joints + 4  */
   float arm_length;        /* L; link length = L / n_joints            (R16)*/
   float h_s;               /* sampling time                            (R16)*/

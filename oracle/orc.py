@@ -52,8 +52,11 @@ class OrcConfig(C.Structure):
                 ("seed", C.c_uint64), ("policy", C.c_int32), ("policy_param", C.c_uint64)]
 
 
+MODEL = {"arm": 0, "lg1": 1}
+
+
 class OrcModel(C.Structure):
-    _fields_ = [("n_joints", C.c_int32), ("arm_length", C.c_float), ("h_s", C.c_float),
+    _fields_ = [("model", C.c_int32), ("n_joints", C.c_int32), ("arm_length", C.c_float), ("h_s", C.c_float),
                 ("sigma_theta", C.c_float), ("sigma_pos", C.c_float), ("sigma_vel", C.c_float),
                 ("sigma_cam", C.c_float), ("sigma_theta_meas", C.c_float)]
 
@@ -147,13 +150,14 @@ class Model:
     sigma_vel: float = 0.1
     sigma_cam: float = 0.1
     sigma_theta_meas: float = 0.1
+    kind: str = "arm"          # "arm" | "lg1" (1-D linear-Gaussian: one joint + its sensor)
 
     @property
     def d(self) -> int:
-        return self.n_joints + 4
+        return 1 if self.kind == "lg1" else self.n_joints + 4
 
     def c(self) -> OrcModel:
-        return OrcModel(self.n_joints, self.arm_length, self.h_s, self.sigma_theta, self.sigma_pos,
+        return OrcModel(MODEL[self.kind], self.n_joints, self.arm_length, self.h_s, self.sigma_theta, self.sigma_pos,
                         self.sigma_vel, self.sigma_cam, self.sigma_theta_meas)
 
 

@@ -13,11 +13,11 @@ import os
 HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.environ.get("PF_LIB") or os.path.join(HERE, "libpf_b200.so")   # PF_LIB: dev A/B builds
 
-PF_OK, PF_EINVAL, PF_ENOMEM, PF_ECUDA, PF_ESTATE, PF_EUNSUPPORTED = 0, -1, -2, -3, -5, -6
+PF_OK, PF_EINVAL, PF_ENOMEM, PF_ECUDA, PF_ESTATE, PF_EUNSUPPORTED, PF_ETIMEOUT = 0, -1, -2, -3, -5, -6, -7
 PF_TOPO_NONE, PF_TOPO_RING, PF_TOPO_TORUS2D, PF_TOPO_ALL2ALL = 0, 1, 2, 3
 PF_RESAMPLE_RWS, PF_RESAMPLE_VOSE = 0, 1
 PF_POLICY_ALWAYS, PF_POLICY_ESS, PF_POLICY_FREQ = 0, 1, 2
-PF_MODEL_ARM_PLANAR = 0
+PF_MODEL_ARM_PLANAR, PF_MODEL_LINEAR_GAUSS_1D = 0, 1
 PF_DEVICE_INPUTS = 1
 
 ENTRY_POINTS = [

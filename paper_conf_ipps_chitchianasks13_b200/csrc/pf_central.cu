@@ -282,16 +282,16 @@ __global__ void __launch_bounds__(256) cz_draw_debug(const CentralParams C, cons
     anc[j] = static_cast<int>(central_ancestor(C, Q, tiles, ua[j], ub[j]));
 }
 
-template <int NJ>
+template <class Model>
 __global__ void __launch_bounds__(256) cz_step(const CentralParams C) {
-  constexpr int D = NJ + 4;
-  __shared__ float z_s[NJ + 2];
-  __shared__ float hsu_s[NJ > 0 ? NJ : 1];
+  constexpr int D = Model::D, ZD = Model::ZD, UD = Model::UD;
+  __shared__ float z_s[ZD];
+  __shared__ float hsu_s[UD];
   __shared__ u64 red[32];
   __shared__ unsigned int s_last;
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  if (tid < NJ + 2) z_s[tid] = C.z ? C.z[tid] : C.zin[tid];
-  if (tid < NJ) hsu_s[tid] = C.mc.hs * (C.u ? C.u[tid] : C.uin[tid]);
+  if (tid < ZD) z_s[tid] = C.z ? C.z[tid] : C.zin[tid];
+  if (tid < UD) hsu_s[tid] = C.mc.hs * (C.u ? C.u[tid] : C.uin[tid]);   // control term h_s u_i (F8)
   __syncthreads();
   const long long M = C.M;
   const int tiles = static_cast<int>(M / kCentralTile);
@@ -310,10 +310,10 @@ __global__ void __launch_bounds__(256) cz_step(const CentralParams C) {
     const float* xa = C.in + a;
     auto x = [xa, M](int c) { return __ldg(xa + c * M); };
     NoiseGen gen{p, C.k, C.rk, u32x4{0u, 0u, b0.z, b0.w}};
-    ArmAcc A;
+    typename Model::Acc A;
     float* out = C.out + i;
-    SampleStream<NJ, 0>::run(C.mc, hsu_s, z_s, x, gen, A, [out, M](int c, float v) { out[c * M] = v; });
-    const float l = arm_finish(C.mc, z_s, A);
+    SampleStream<Model, 0>::run(C.mc, hsu_s, z_s, x, gen, A, [out, M](int c, float v) { out[c * M] = v; });
+    const float l = Model::finish(C.mc, z_s, A);
     out[D * M] = l;
     const u64 key = order_key(l, p);
     best = key > best ? key : best;
@@ -369,26 +369,27 @@ void vose_table(const CentralParams& c, cudaStream_t s) {
   vz_table<<<g2, 256, 0, s>>>(c);
 }
 
-template <int NJ>
-cudaError_t central_step_nj(const CentralParams& c, int grid, cudaStream_t s) {
+template <class Model>
+cudaError_t central_step_m(const CentralParams& c, int grid, cudaStream_t s) {
   const int tiles = static_cast<int>(c.M / kCentralTile);
   if (!c.first && !c.publish) {
-    cz_tile_scan<<<tiles, kScanThreads, 0, s>>>(c.in + static_cast<long long>(NJ + 4) * c.M, c.record_prev, c.cl,
+    cz_tile_scan<<<tiles, kScanThreads, 0, s>>>(c.in + static_cast<long long>(Model::D) * c.M, c.record_prev, c.cl,
                                                 c.tile_sum);
     cz_tile_prefix<<<1, 1024, 0, s>>>(c.tile_sum, c.tile_incl, tiles);
     if (c.vose) vose_table(c, s);
   }
-  cz_step<NJ><<<grid, 256, 0, s>>>(c);
+  cz_step<Model><<<grid, 256, 0, s>>>(c);
   return cudaGetLastError();
 }
 
 }  // namespace
 
-cudaError_t central_step(int nj, const CentralParams& c, int grid, cudaStream_t s) {
+cudaError_t central_step(int model, int nj, const CentralParams& c, int grid, cudaStream_t s) {
+  if (model == MODEL_LINEAR_GAUSS_1D) return central_step_m<LinearGauss1D>(c, grid, s);
   switch (nj) {
-    case 2: return central_step_nj<2>(c, grid, s);
-    case 5: return central_step_nj<5>(c, grid, s);
-    case 28: return central_step_nj<28>(c, grid, s);
+    case 2: return central_step_m<ArmPlanar<2>>(c, grid, s);
+    case 5: return central_step_m<ArmPlanar<5>>(c, grid, s);
+    case 28: return central_step_m<ArmPlanar<28>>(c, grid, s);
     default: return cudaErrorInvalidValue;
   }
 }
@@ -403,14 +404,18 @@ cudaError_t central_resample_debug(const CentralParams& c, const uint32_t* q, co
   return cudaGetLastError();
 }
 
-int central_grid(int nj, int sms) {
+int central_grid(int model, int nj, int sms) {
   int bps = 0;
   cudaError_t e = cudaErrorInvalidValue;
-  switch (nj) {
-    case 2: e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, cz_step<2>, 256, 0); break;
-    case 5: e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, cz_step<5>, 256, 0); break;
-    case 28: e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, cz_step<28>, 256, 0); break;
-    default: break;
+  if (model == MODEL_LINEAR_GAUSS_1D) {
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, cz_step<LinearGauss1D>, 256, 0);
+  } else {
+    switch (nj) {
+      case 2: e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, cz_step<ArmPlanar<2>>, 256, 0); break;
+      case 5: e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, cz_step<ArmPlanar<5>>, 256, 0); break;
+      case 28: e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, cz_step<ArmPlanar<28>>, 256, 0); break;
+      default: break;
+    }
   }
   return (e == cudaSuccess && bps > 0) ? bps * sms : 0;
 }

@@ -4,14 +4,14 @@
 
 #include <cstdint>
 
-#include "pf_device.cuh"
+#include "pf_model.cuh"
 
 namespace pf {
 
 constexpr int kCentralTile = 4096;   // particles per scan tile (M must be a multiple)
 
 struct CentralParams {
-  ArmConsts mc;
+  ModelConsts mc;           // model constants (pf_model.cuh)
   const float* in;          // [D+1][M] weighted set of step k-1 (buffer (k-1)&1)
   float* out;               // [D+1][M] step k (buffer k&1)
   long long M;
@@ -51,11 +51,12 @@ struct CentralParams {
 // (<= M Q <= M^2 2^22) stay below 2^64.
 constexpr long long kCentralVoseMax = 1ll << 20;
 
-cudaError_t central_step(int nj, const CentralParams& c, int grid, cudaStream_t s);
+// model: pf_model_id; nj: the arm's n_joints (2, 5, 28), ignored for the 1-D linear-Gaussian model
+cudaError_t central_step(int model, int nj, const CentralParams& c, int grid, cudaStream_t s);
 // test hook: RWS / Vose ancestors over all M slots from integer weights q [M]
 // and uniforms ua, ub [M] (device); the Vose table is left in c.prob / c.alias
 cudaError_t central_resample_debug(const CentralParams& c, const uint32_t* q, const uint32_t* ua, const uint32_t* ub,
                                    int* anc, cudaStream_t s);
-int central_grid(int nj, int sms);
+int central_grid(int model, int nj, int sms);
 
 }  // namespace pf

@@ -33,6 +33,7 @@
 #include <type_traits>
 
 #include "pf_device.cuh"
+#include "pf_model.cuh"
 
 namespace pf {
 
@@ -50,19 +51,27 @@ constexpr int kRecordSeq = 127;
 
 // Peer transport (world > 1 on one node, NVLink/NVSwitch peer memory): every
 // rank's runtime owns a small "peer block" that the other ranks write into:
-// [kMaxRanks] u64 step flags, then [kMaxRanks][kPeerRec] float records.
+// [kMaxRanks] u64 rendezvous flags, then [2][kMaxRanks][kPeerRec] float
+// records, then [2][kMaxRanks][kPeerPool] float All-to-All pool rows — the
+// records and pool rows double-buffered by the parity of the rendezvous
+// number (see the ordering argument at the rendezvous and DESIGN.md §8).
 constexpr int kMaxRanks = 8;
 constexpr int kPeerRec = 40;   // 4 + d <= 36 floats, padded
 constexpr int kPeerPool = 32 * 34;   // All-to-All: t <= 32 entries of E = d + 2 <= 34 floats
+constexpr size_t kPeerBlockUsed =
+    sizeof(unsigned long long) * kMaxRanks + sizeof(float) * 2 * kMaxRanks * (kPeerRec + kPeerPool);
+// record word 3 (a status, 0 = ok): the rendezvous timed out (a rank did not
+// arrive within peer_timeout_ns) — the record is not the global estimate
+constexpr uint32_t kStatusPeerTimeout = 1u;
 
 struct StepParams {
-  ArmConsts mc;
-  ArmConsts2 mc2;          // mc with every field duplicated (packed f32x2 operands)
+  ModelConsts mc;          // model constants (pf_model.cuh)
+  ModelConsts2 mc2;        // mc with every field duplicated (packed f32x2 operands)
   float* parts;            // [n_local][D+1][M] blocked SoA (row D = log-weight)
   const float* mb_prev;    // mailbox parity (k-1)&1 : [n_ext][tt][E]
   float* mb_cur;           // mailbox parity k&1
-  const float* z;          // [NJ+2] device, or nullptr: use zin
-  const float* u;          // [NJ]   device, or nullptr: use uin
+  const float* z;          // [ZD] device, or nullptr: use zin
+  const float* u;          // [UD] device, or nullptr: use uin
   u64* key_cur;            // global best key of this step (0 on entry)
   u64* key_next;           // reset to 0 for the next step
   unsigned int* counter;   // CTA completion counter (0 on entry, reset by the last CTA)
@@ -91,6 +100,8 @@ struct StepParams {
   unsigned char* peer_blk[kMaxRanks];
   int rank, world;
   long long mb_parity;     // floats per mailbox parity (n_ext * tt * E), same on every rank
+  unsigned long long rv;   // peer rendezvous number of this launch (>= 1, +1 per peer-mode launch on every rank)
+  unsigned long long peer_timeout_ns;   // give up waiting at the rendezvous after this long (status word)
   float zin[32];           // step inputs carried by the launch itself (host-input mode)
   float uin[32];
 };
@@ -150,24 +161,23 @@ __device__ __forceinline__ unsigned long long tl_now() {
 #endif
 
 // ------------------------------------------------------- configuration
-// NJ joints (D = NJ + 4), M particles per sub-filter, resampler RES; a group
+// Model (pf_model.cuh: D state components, the sample / weight hooks), M
+// particles per sub-filter, resampler RES; a group
 // of GW warps owns one sub-filter; S groups per CTA; NSTAGE TMA stages per
 // group; the per-particle sample/weight loop over a thread's P slots is
 // unrolled UNR times (P for full unrolling; 1 keeps one copy of the
 // ~10–40 KB per-particle code in the instruction cache).
-#ifndef PF_CHUNK_MIN_D
-#define PF_CHUNK_MIN_D 16
-#endif
 #ifndef PF_X2_DEFAULT
 #define PF_X2_DEFAULT 1
 #endif
-template <int NJ_, int M_, int RES_, int GW_, int S_, int NSTAGE_, int UNR_, int MINB_, int EARLY_ = 0,
+template <class Model_, int M_, int RES_, int GW_, int S_, int NSTAGE_, int UNR_, int MINB_, int EARLY_ = 0,
           int X2_ = PF_X2_DEFAULT>
 struct KCfg {
+  using Model = Model_;
   static constexpr int EARLY = EARLY_;       // start the next TMA load right after the sample loop
-  static constexpr int NJ = NJ_, M = M_, RES = RES_, GW = GW_, S = S_, NSTAGE = NSTAGE_, UNR = UNR_;
+  static constexpr int M = M_, RES = RES_, GW = GW_, S = S_, NSTAGE = NSTAGE_, UNR = UNR_;
   static constexpr int MINB = MINB_;         // __launch_bounds__ min CTAs per SM (register cap)
-  static constexpr int D = NJ + 4;
+  static constexpr int D = Model::D;
   static constexpr int E = D + 2;            // mailbox entry: [logw, index bits, x_0..x_{D-1}]
   static constexpr int T = 32 * GW;          // threads per group
   static constexpr int P = M / T;            // particles per thread
@@ -175,10 +185,7 @@ struct KCfg {
   static constexpr bool SCAN32 = (M <= 512);  // Q <= M 2^22 fits 32 bits
   static constexpr bool STAGED = UNR < P;    // rolled sample loop: per-slot values via smem
   static constexpr bool X2 = X2_ && (P % 2 == 0);   // sample two particles at once (packed f32x2)
-  // large states (the high-DOF arm): the joint chain runs as a loop over
-  // chunks of four joints instead of being unrolled d times, so the
-  // per-particle code fits the instruction cache (ncu: no_instruction stalls)
-  static constexpr bool CHUNKED = D > PF_CHUNK_MIN_D;
+  static constexpr bool CHUNKED = Model::CHUNKED;   // runtime loop over joint chunks (pf_model.cuh)
   static_assert(P >= 1 && P * T == M, "M must be a multiple of the group size");
   static_assert(P <= 32, "exclusion masks are 32-bit");
   static_assert(S >= 1 && S <= 15, "named barriers 1..S");
@@ -197,7 +204,7 @@ struct KCfg {
   static constexpr size_t g_bar = g_misc + sizeof(int) * GW * 2 * KMAX;          // u64 [2] + next [2]
   static constexpr size_t group_bytes = (g_bar + 32 + 127) / 128 * 128;
   // per-CTA
-  static constexpr size_t c_zin = 0;          // float [64]: z (NJ+2), h_s u (NJ)
+  static constexpr size_t c_zin = 0;          // float [64]: z (ZD), h_s u (UD)
   static constexpr size_t c_zin2 = 256;       // f2 [64]: the same, each value duplicated (packed operands)
   static constexpr size_t c_groups = 768;
   static constexpr size_t smem = c_groups + S * group_bytes;
@@ -581,19 +588,20 @@ struct NoiseGen {
   }
 };
 
-// Streamed sample + weight of one particle (F8–F10), Box–Muller pair by
-// pair; out(c, v) stores component c of the new state.
-template <int NJ, int QP>
+// Streamed sample + weight of one particle (F8–F10) through the model's
+// take<c> hooks, Box–Muller pair by pair; out(c, v) stores component c of
+// the new state.
+template <class Model, int QP>
 struct SampleStream {
-  static constexpr int D = NJ + 4;
+  static constexpr int D = Model::D;
   template <typename X, typename O>
-  __device__ __forceinline__ static void run(const ArmConsts& mc, const float* hsu, const float* z, const X& x,
-                                             NoiseGen& gen, ArmAcc& A, const O& out) {
+  __device__ __forceinline__ static void run(const ModelConsts& mc, const float* hsu, const float* z, const X& x,
+                                             NoiseGen& gen, typename Model::Acc& A, const O& out) {
     float z0, z1;
     gen.template pair<QP>(z0, z1);
-    out(2 * QP, arm_sample_take<NJ, 2 * QP>(mc, hsu, z, x, z0, A));
-    if constexpr (2 * QP + 1 < D) out(2 * QP + 1, arm_sample_take<NJ, 2 * QP + 1>(mc, hsu, z, x, z1, A));
-    if constexpr (QP + 1 < (D + 1) / 2) SampleStream<NJ, QP + 1>::run(mc, hsu, z, x, gen, A, out);
+    out(2 * QP, Model::template take<2 * QP>(mc, hsu, z, x, z0, A));
+    if constexpr (2 * QP + 1 < D) out(2 * QP + 1, Model::template take<2 * QP + 1>(mc, hsu, z, x, z1, A));
+    if constexpr (QP + 1 < (D + 1) / 2) SampleStream<Model, QP + 1>::run(mc, hsu, z, x, gen, A, out);
   }
 };
 
@@ -615,113 +623,81 @@ struct NoiseGen2 {
   }
 };
 
-template <int NJ, int QP>
+template <class Model, int QP>
 struct SampleStream2 {
-  static constexpr int D = NJ + 4;
+  static constexpr int D = Model::D;
   template <typename X, typename O>
-  __device__ __forceinline__ static void run(const ArmConsts2& mc, const f2* hsu2, const f2* z2, const X& x,
-                                             NoiseGen2& gen, ArmAcc2& A, const O& out) {
+  __device__ __forceinline__ static void run(const ModelConsts2& mc, const f2* hsu2, const f2* z2, const X& x,
+                                             NoiseGen2& gen, typename Model::Acc2& A, const O& out) {
     f2 z0, z1;
     gen.template pair<QP>(z0, z1);
-    out(2 * QP, arm_sample_take2<NJ, 2 * QP>(mc, hsu2, z2, x, z0, A));
-    if constexpr (2 * QP + 1 < D) out(2 * QP + 1, arm_sample_take2<NJ, 2 * QP + 1>(mc, hsu2, z2, x, z1, A));
-    if constexpr (QP + 1 < (D + 1) / 2) SampleStream2<NJ, QP + 1>::run(mc, hsu2, z2, x, gen, A, out);
+    out(2 * QP, Model::template take2<2 * QP>(mc, hsu2, z2, x, z0, A));
+    if constexpr (2 * QP + 1 < D) out(2 * QP + 1, Model::template take2<2 * QP + 1>(mc, hsu2, z2, x, z1, A));
+    if constexpr (QP + 1 < (D + 1) / 2) SampleStream2<Model, QP + 1>::run(mc, hsu2, z2, x, gen, A, out);
   }
 };
 
 // The same streamed sample + weight as SampleStream / SampleStream2 for large
-// states, with the middle of the joint chain as a runtime loop: pair 0
-// (components 0, 1; block 0 words 2-3 supplied) static, then chunks of four
-// joints 2 + 4i .. 5 + 4i that use exactly Philox block i + 1 (words 4-7 of
-// the chunk), then the remaining components static from pair 1 + 2 NC on.
-// One copy of four joints' code instead of d (instruction cache), identical
-// arithmetic in the same order.
-template <int NJ>
+// states (Model::CHUNKED), with the middle of the chain as a runtime loop:
+// pair 0 (components 0, 1; block 0 words 2-3 supplied) static, then NC
+// chunks of four components 2 + 4i .. 5 + 4i (Model::joint) that use exactly
+// Philox block i + 1 (words 4-7 of the chunk), then the remaining components
+// static from pair 1 + 2 NC on.  One copy of four components' code instead of
+// d (instruction cache), identical arithmetic in the same order.
+template <class Model>
 struct SampleChunked {
-  static constexpr int D = NJ + 4;
-  static constexpr int NC = NJ >= 6 ? (NJ - 2) / 4 : 0;   // chunks of four joints
-  template <typename X>
-  __device__ __forceinline__ static void joint(int c, const ArmConsts& mc, const float* hsu, const float* z, const X& x,
-                                               float xi, ArmAcc& A, float& th) {
-    th = __fmaf_rn(mc.s_th, xi, x(c) + hsu[c]);
-    A.phi = A.phi + th;
-    sincos_c(A.phi, A.s, A.c);
-    A.px = __fmaf_rn(mc.lj, A.c, A.px);
-    A.py = __fmaf_rn(mc.lj, A.s, A.py);
-    const float r = (z[2 + c] - th) * mc.inv_thm;
-    A.acc = __fmaf_rn(r, r, A.acc);   // c >= 2: never the first joint
-  }
+  static constexpr int NC = Model::NC;
   template <typename X, typename O>
-  __device__ __forceinline__ static void run(const ArmConsts& mc, const float* hsu, const float* z, const X& x,
-                                             NoiseGen& gen, ArmAcc& A, const O& out) {
+  __device__ __forceinline__ static void run(const ModelConsts& mc, const float* hsu, const float* z, const X& x,
+                                             NoiseGen& gen, typename Model::Acc& A, const O& out) {
     {
       float z0, z1;
       gen.template pair<0>(z0, z1);
-      out(0, arm_sample_take<NJ, 0>(mc, hsu, z, x, z0, A));
-      out(1, arm_sample_take<NJ, 1>(mc, hsu, z, x, z1, A));
+      out(0, Model::template take<0>(mc, hsu, z, x, z0, A));
+      out(1, Model::template take<1>(mc, hsu, z, x, z1, A));
     }
 #pragma unroll 1
     for (int i = 0; i < NC; ++i) {
       const int c = 2 + 4 * i;
       const u32x4 b = philox4x32_10_rk(gen.p, gen.k, 0u, static_cast<uint32_t>(i + 1), gen.rk);
-      float n0, n1, n2, n3, th;
+      float n0, n1, n2, n3;
       normal_pair(b.x, b.y, n0, n1);
       normal_pair(b.z, b.w, n2, n3);
-      joint(c, mc, hsu, z, x, n0, A, th);
-      out(c, th);
-      joint(c + 1, mc, hsu, z, x, n1, A, th);
-      out(c + 1, th);
-      joint(c + 2, mc, hsu, z, x, n2, A, th);
-      out(c + 2, th);
-      joint(c + 3, mc, hsu, z, x, n3, A, th);
-      out(c + 3, th);
+      out(c, Model::joint(c, mc, hsu, z, x, n0, A));
+      out(c + 1, Model::joint(c + 1, mc, hsu, z, x, n1, A));
+      out(c + 2, Model::joint(c + 2, mc, hsu, z, x, n2, A));
+      out(c + 3, Model::joint(c + 3, mc, hsu, z, x, n3, A));
     }
-    SampleStream<NJ, 1 + 2 * NC>::run(mc, hsu, z, x, gen, A, out);
+    SampleStream<Model, 1 + 2 * NC>::run(mc, hsu, z, x, gen, A, out);
   }
 };
 
-template <int NJ>
+template <class Model>
 struct SampleChunked2 {
-  static constexpr int D = NJ + 4;
-  static constexpr int NC = NJ >= 6 ? (NJ - 2) / 4 : 0;
-  template <typename X>
-  __device__ __forceinline__ static void joint(int c, const ArmConsts2& mc, const f2* hsu2, const f2* z2, const X& x,
-                                               f2 xi, ArmAcc2& A, f2& th) {
-    th = fma2(mc.s_th, xi, add2(x(c), hsu2[c]));
-    A.phi = add2(A.phi, th);
-    sincos_c2(A.phi, A.s, A.c);
-    A.px = fma2(mc.lj, A.c, A.px);
-    A.py = fma2(mc.lj, A.s, A.py);
-    const f2 r = mul2(sub2(z2[2 + c], th), mc.inv_thm);
-    A.acc = fma2(r, r, A.acc);   // c >= 2
-  }
+  static constexpr int NC = Model::NC;
   template <typename X, typename O>
-  __device__ __forceinline__ static void run(const ArmConsts2& mc, const f2* hsu2, const f2* z2, const X& x,
-                                             NoiseGen2& gen, ArmAcc2& A, const O& out) {
+  __device__ __forceinline__ static void run(const ModelConsts2& mc, const f2* hsu2, const f2* z2, const X& x,
+                                             NoiseGen2& gen, typename Model::Acc2& A, const O& out) {
     {
       f2 z0, z1;
       gen.template pair<0>(z0, z1);
-      out(0, arm_sample_take2<NJ, 0>(mc, hsu2, z2, x, z0, A));
-      out(1, arm_sample_take2<NJ, 1>(mc, hsu2, z2, x, z1, A));
+      out(0, Model::template take2<0>(mc, hsu2, z2, x, z0, A));
+      out(1, Model::template take2<1>(mc, hsu2, z2, x, z1, A));
     }
 #pragma unroll 1
     for (int i = 0; i < NC; ++i) {
       const int c = 2 + 4 * i;
       const u32x4 ba = philox4x32_10_rk(gen.pa, gen.k, 0u, static_cast<uint32_t>(i + 1), gen.rk);
       const u32x4 bb = philox4x32_10_rk(gen.pb, gen.k, 0u, static_cast<uint32_t>(i + 1), gen.rk);
-      f2 n0, n1, n2, n3, th;
+      f2 n0, n1, n2, n3;
       normal_pair2(ba.x, ba.y, bb.x, bb.y, n0, n1);
       normal_pair2(ba.z, ba.w, bb.z, bb.w, n2, n3);
-      joint(c, mc, hsu2, z2, x, n0, A, th);
-      out(c, th);
-      joint(c + 1, mc, hsu2, z2, x, n1, A, th);
-      out(c + 1, th);
-      joint(c + 2, mc, hsu2, z2, x, n2, A, th);
-      out(c + 2, th);
-      joint(c + 3, mc, hsu2, z2, x, n3, A, th);
-      out(c + 3, th);
+      out(c, Model::joint2(c, mc, hsu2, z2, x, n0, A));
+      out(c + 1, Model::joint2(c + 1, mc, hsu2, z2, x, n1, A));
+      out(c + 2, Model::joint2(c + 2, mc, hsu2, z2, x, n2, A));
+      out(c + 3, Model::joint2(c + 3, mc, hsu2, z2, x, n3, A));
     }
-    SampleStream2<NJ, 1 + 2 * NC>::run(mc, hsu2, z2, x, gen, A, out);
+    SampleStream2<Model, 1 + 2 * NC>::run(mc, hsu2, z2, x, gen, A, out);
   }
 };
 
@@ -757,11 +733,18 @@ __device__ void peer_halo_rows(const StepParams& P) {   // whole CTA (the last o
 __device__ __forceinline__ unsigned long long* peer_flags(unsigned char* blk) {
   return reinterpret_cast<unsigned long long*>(blk);
 }
-__device__ __forceinline__ float* peer_rec(unsigned char* blk, int r) {
-  return reinterpret_cast<float*>(blk + sizeof(unsigned long long) * kMaxRanks) + r * kPeerRec;
+// record / pool row of rank r in buffer par (= rendezvous number & 1)
+__device__ __forceinline__ float* peer_rec(unsigned char* blk, int par, int r) {
+  return reinterpret_cast<float*>(blk + sizeof(unsigned long long) * kMaxRanks) + (par * kMaxRanks + r) * kPeerRec;
 }
-__device__ __forceinline__ float* peer_pool(unsigned char* blk, int r) {
-  return peer_rec(blk, kMaxRanks) + r * kPeerPool;
+__device__ __forceinline__ float* peer_pool(unsigned char* blk, int par, int r) {
+  return reinterpret_cast<float*>(blk + sizeof(unsigned long long) * kMaxRanks) + 2 * kMaxRanks * kPeerRec +
+         (par * kMaxRanks + r) * kPeerPool;
+}
+__device__ __forceinline__ unsigned long long global_ns() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
 }
 
 // Best t of the union of two descending lists held by lanes 0..t-1 (run list
@@ -878,12 +861,13 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
 #ifdef PF_TIMELINE
   if (threadIdx.x == 0) atomicMin(&pf_tl2[0], tl_now());
 #endif
-  constexpr int NJ = C::NJ, M = C::M, D = C::D, E = C::E, GW = C::GW, PP = C::P;
+  using Model = typename C::Model;
+  constexpr int ZD = Model::ZD, UD = Model::UD, M = C::M, D = C::D, E = C::E, GW = C::GW, PP = C::P;
   extern __shared__ __align__(128) unsigned char smem[];
   float* z_s = reinterpret_cast<float*>(smem + C::c_zin);
-  float* hsu_s = z_s + NJ + 2;
+  float* hsu_s = z_s + ZD;
   f2* z2_s = reinterpret_cast<f2*>(smem + C::c_zin2);
-  f2* hsu2_s = z2_s + NJ + 2;
+  f2* hsu2_s = z2_s + ZD;
 
   const int g = threadIdx.x / C::T;
   unsigned char* gs = smem + C::c_groups + g * C::group_bytes;
@@ -950,12 +934,12 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
     if (gid0 < P.n_local) pending = atomicAdd(P.work, 1u);
   }
   if (do_sample) {
-    if (threadIdx.x < NJ + 2) {
+    if (threadIdx.x < ZD) {
       const float v = P.z ? P.z[threadIdx.x] : P.zin[threadIdx.x];
       z_s[threadIdx.x] = v;
       z2_s[threadIdx.x] = bc(v);
     }
-    if (threadIdx.x < NJ) {
+    if (threadIdx.x < UD) {   // control term h_s u_i (F8)
       const float v = P.mc.hs * (P.u ? P.u[threadIdx.x] : P.uin[threadIdx.x]);
       hsu_s[threadIdx.x] = v;
       hsu2_s[threadIdx.x] = bc(v);
@@ -1269,17 +1253,17 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
         float* outb = gblk + sb;
         NoiseGen2 gen{pbase + static_cast<uint32_t>(sa), pbase + static_cast<uint32_t>(sb), P.k, P.rk,
                       u32x4{0u, 0u, za2, za3}, u32x4{0u, 0u, zb2, zb3}};
-        ArmAcc2 A;
+        typename Model::Acc2 A;
         auto store2 = [outa, outb](int c, f2 v) {
           outa[c * M] = lo2(v);
           outb[c * M] = hi2(v);
         };
         if constexpr (C::CHUNKED) {
-          SampleChunked2<NJ>::run(P.mc2, hsu2_s, z2_s, x, gen, A, store2);
+          SampleChunked2<Model>::run(P.mc2, hsu2_s, z2_s, x, gen, A, store2);
         } else {
-          SampleStream2<NJ, 0>::run(P.mc2, hsu2_s, z2_s, x, gen, A, store2);
+          SampleStream2<Model, 0>::run(P.mc2, hsu2_s, z2_s, x, gen, A, store2);
         }
-        f2 l = arm_finish2(P.mc2, z2_s, A);
+        f2 l = Model::finish2(P.mc2, z2_s, A);
         if (!resampled) l = add2(pk(c0, c1), l);   // F12
         outa[D * M] = lo2(l);
         outb[D * M] = hi2(l);
@@ -1316,10 +1300,10 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
         auto x = [xa](int c) { return xa[c * M]; };
         float* out = gblk + s;
         NoiseGen gen{pbase + static_cast<uint32_t>(s), P.k, P.rk, u32x4{0u, 0u, z2, z3}};
-        ArmAcc A;
+        typename Model::Acc A;
         // (one particle per thread: the unrolled chain measured as fast as the chunked one)
-        SampleStream<NJ, 0>::run(P.mc, hsu_s, z_s, x, gen, A, [out](int c, float v) { out[c * M] = v; });
-        float l = arm_finish(P.mc, z_s, A);
+        SampleStream<Model, 0>::run(P.mc, hsu_s, z_s, x, gen, A, [out](int c, float v) { out[c * M] = v; });
+        float l = Model::finish(P.mc, z_s, A);
         if (!resampled) l = cr + l;   // F12
         out[D * M] = l;
         reinterpret_cast<float*>(bzw_s)[2 * s] = l;   // own slot, after its Philox words were read
@@ -1468,42 +1452,58 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
         // (device-side rendezvous over NVLink), then the exact max over the
         // world records (the all-gather + pf_reduce_records of the NCCL path)
         const bool a2a = P.topo == TOPO_A2A && P.t > 0;
+        const int par = static_cast<int>(P.rv & 1ull);
         if (a2a) {
           __syncthreads();   // the local pool row is complete
           const float* lp = P.mb_cur + P.pool_local_row * P.tt * E;
           for (int i = tid; i < P.world * P.t * E; i += blockDim.x) {
             const int r = i / (P.t * E), e = i - r * (P.t * E);
-            peer_pool(P.peer_blk[r], P.rank)[e] = __ldcg(lp + e);
+            peer_pool(P.peer_blk[r], par, P.rank)[e] = __ldcg(lp + e);
           }
         } else {
           peer_halo_rows<E>(P);
         }
         if (tid < D) {
           const float v = __ldcg(blk + tid * M);
-          for (int r = 0; r < P.world; ++r) peer_rec(P.peer_blk[r], P.rank)[4 + tid] = v;
+          for (int r = 0; r < P.world; ++r) peer_rec(P.peer_blk[r], par, P.rank)[4 + tid] = v;
         }
         if (tid == 0) {
           const float r4[4] = {__uint_as_float(static_cast<uint32_t>(key)),
                                __uint_as_float(static_cast<uint32_t>(key >> 32)),
                                unord_f32(static_cast<uint32_t>(key >> 32)), 0.0f};
           for (int r = 0; r < P.world; ++r)
-            for (int c = 0; c < 4; ++c) peer_rec(P.peer_blk[r], P.rank)[c] = r4[c];
+            for (int c = 0; c < 4; ++c) peer_rec(P.peer_blk[r], par, P.rank)[c] = r4[c];
         }
         __threadfence_system();
         __syncthreads();
-        const unsigned long long kk = P.k;
+        // Rendezvous number rv (not the step number: flags only grow, also
+        // across pf_set_particles).  Ordering: a rank writes the records /
+        // pool rows of rendezvous rv into buffer rv & 1 BEFORE raising flag
+        // rv, and starts rendezvous rv + 1 only after every rank raised flag
+        // rv.  Rank B raises flag rv + 1 only after its rendezvous-rv reads
+        // are done (they precede its kernel's completion), so rank A's writes
+        // of rendezvous rv + 2 into buffer rv & 1 (issued after A passed
+        // rendezvous rv + 1) cannot overwrite anything B still reads.
+        const unsigned long long kk = P.rv;
+        int late = 0;
         if (tid < P.world) {
           unsigned long long* f = peer_flags(P.peer_blk[tid]) + P.rank;
           asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(f), "l"(kk) : "memory");
           const unsigned long long* mine = peer_flags(P.peer_blk[P.rank]) + tid;
+          const unsigned long long t0 = global_ns();
           unsigned long long seen;
-          do {
+          for (;;) {
             asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(seen) : "l"(mine) : "memory");
-          } while (seen < kk);
+            if (seen >= kk) break;
+            if (global_ns() - t0 > P.peer_timeout_ns) {   // a rank did not arrive: report, do not hang
+              late = 1;
+              break;
+            }
+          }
         }
-        __syncthreads();
+        const bool timed_out = __syncthreads_or(late) != 0;
         if (tid < 32) {
-          const float* rec0 = peer_rec(P.peer_blk[P.rank], 0);
+          const float* rec0 = peer_rec(P.peer_blk[P.rank], par, 0);
           u64 k2 = 0ull;
           if (tid < P.world)
             k2 = static_cast<u64>(__float_as_uint(__ldcv(rec0 + tid * kPeerRec))) |
@@ -1511,7 +1511,8 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
           const u64 w = warp_max_u64(k2);
           const int src = __ffs(__ballot_sync(0xFFFFFFFFu, tid < P.world && k2 == w)) - 1;
           for (int c = tid; c < 4 + D; c += 32) {
-            const float v = __ldcv(rec0 + src * kPeerRec + c);
+            const float v = c == 3 ? __uint_as_float(timed_out ? kStatusPeerTimeout : 0u)
+                                   : __ldcv(rec0 + src * kPeerRec + c);
             for (int o = 0; o < 3; ++o)
               if (outs[o]) outs[o][c] = v;
           }
@@ -1523,7 +1524,7 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
               int be = -1;
               for (int e = tid; e < P.world * P.t; e += 32) {
                 const int r = e / P.t, jj = e - r * P.t;
-                const float* en = peer_pool(P.peer_blk[P.rank], r) + jj * E;
+                const float* en = peer_pool(P.peer_blk[P.rank], par, r) + jj * E;
                 const u64 kk2 = order_key(__ldcv(en), __float_as_uint(__ldcv(en + 1)));
                 if (kk2 < prev && kk2 > best) {
                   best = kk2;
@@ -1535,7 +1536,7 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
               const int bsel = __shfl_sync(0xFFFFFFFFu, be, own < 0 ? 0 : own);
               if (own >= 0) {
                 const int r = bsel / P.t, jj = bsel - r * P.t;
-                const float* en = peer_pool(P.peer_blk[P.rank], r) + jj * E;
+                const float* en = peer_pool(P.peer_blk[P.rank], par, r) + jj * E;
                 for (int c = tid; c < E; c += 32) out[jb * E + c] = __ldcv(en + c);
               }
               prev = g2;

@@ -103,6 +103,8 @@ __global__ void mean_final_kernel(const double* __restrict__ partials, int count
 
 cudaError_t mean_partials(const MeanParams& mp, cudaStream_t s) {
   switch (mp.d) {
+    case 1: mean_partial_kernel<1><<<kMeanGrid, kMeanThreads, 0, s>>>(mp.parts, mp.n_blocks, mp.m, mp.row, mp.record,
+                                                                       mp.partials); break;   // linear-Gaussian model
     case 6: mean_partial_kernel<6><<<kMeanGrid, kMeanThreads, 0, s>>>(mp.parts, mp.n_blocks, mp.m, mp.row, mp.record,
                                                                        mp.partials); break;
     case 9: mean_partial_kernel<9><<<kMeanGrid, kMeanThreads, 0, s>>>(mp.parts, mp.n_blocks, mp.m, mp.row, mp.record,

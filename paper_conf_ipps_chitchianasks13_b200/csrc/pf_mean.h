@@ -11,7 +11,7 @@ struct MeanParams {
   const float* parts;   // weighted set, blocked SoA [n_blocks][d+1][m]
   long long n_blocks;   // sub-filters of the shard (the centralized filter: 1)
   int m;                // particles per block
-  int d;                // state dimension (6, 9 or 32)
+  int d;                // state dimension (1, 6, 9 or 32)
   long long row;        // floats per block, (d+1) m
   const float* record;  // estimate record: record[2] = log-weight of the (global) best particle
   double* partials;     // [kMeanGrid][d+1] scratch

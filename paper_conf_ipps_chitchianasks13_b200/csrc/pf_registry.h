@@ -1,9 +1,10 @@
 // pf_registry.h — table of compiled pf_step_kernel instantiations.
 //
-// Each pf_inst_nj*.cu translation unit instantiates one n_joints value for
-// every m in {32, ..., 1024} and both resamplers (plus alternative mappings
-// of the hottest configurations).  The runtime takes the FIRST entry that
-// matches (n_joints, m, resampler); PF_VARIANT=<i> in the environment selects
+// Each pf_inst_*.cu translation unit instantiates one model (pf_model.cuh:
+// the arm for one n_joints value, or the 1-D linear-Gaussian model) for every
+// m in {32, ..., 1024} and both resamplers (plus alternative mappings of the
+// hottest configurations).  The runtime takes the FIRST entry that matches
+// (model, n_joints, m, resampler); PF_VARIANT=<i> in the environment selects
 // the i-th matching entry instead (tuning knob, default 0).
 #pragma once
 #include <cuda_runtime.h>
@@ -15,7 +16,7 @@ namespace pf {
 struct StepParams;
 
 struct KernelEntry {
-  int nj, m, res;
+  int model, nj, m, res;          // pf_model_id; n_joints (arm) or 1
   int gw, s, nstage, unr, minb;   // warps per group, groups per CTA, TMA stages, sample unroll, min CTAs/SM
   int large;                      // preferred when the shard has >= kLargeNLocal sub-filters
   cudaError_t (*prepare)(int* blocks_per_sm);
@@ -31,22 +32,18 @@ extern const KernelEntry kEntriesNJ5[];
 extern const int kNumEntriesNJ5;
 extern const KernelEntry kEntriesNJ28[];
 extern const int kNumEntriesNJ28;
+extern const KernelEntry kEntriesLG1[];
+extern const int kNumEntriesLG1;
 }  // namespace pf
 
-#define PF_ENTRY(NJ, M, RES, GW, S, NST, UNR, MINB)                                                             \
-  {NJ,                                                                                                    \
-   M,                                                                                                     \
-   RES,                                                                                                   \
-   GW,                                                                                                    \
-   S,                                                                                                     \
-   NST,                                                                                                   \
-   UNR,                                                                                                   \
-   MINB,                                                                                                  \
-   0,                                                                                                     \
-   &StepKernel<KCfg<NJ, M, RES, GW, S, NST, UNR, MINB>>::prepare,                                               \
-   &StepKernel<KCfg<NJ, M, RES, GW, S, NST, UNR, MINB>>::launch,                                                \
-   &StepKernel<KCfg<NJ, M, RES, GW, S, NST, UNR, MINB>>::resample_debug,                                        \
-   StepKernel<KCfg<NJ, M, RES, GW, S, NST, UNR, MINB>>::smem()}
+// one table entry for model type MT (its kId, n_joints NJ)
+#define PF_ENTRY_MT(MT, NJ, LARGE, M, RES, GW, S, NST, UNR, MINB)                                     \
+  {MT::kId, NJ, M, RES, GW, S, NST, UNR, MINB, LARGE,                                               \
+   &StepKernel<KCfg<MT, M, RES, GW, S, NST, UNR, MINB>>::prepare,                                    \
+   &StepKernel<KCfg<MT, M, RES, GW, S, NST, UNR, MINB>>::launch,                                     \
+   &StepKernel<KCfg<MT, M, RES, GW, S, NST, UNR, MINB>>::resample_debug,                             \
+   StepKernel<KCfg<MT, M, RES, GW, S, NST, UNR, MINB>>::smem()}
+#define PF_ENTRY(NJ, M, RES, GW, S, NST, UNR, MINB) PF_ENTRY_MT(ArmPlanar<NJ>, NJ, 0, M, RES, GW, S, NST, UNR, MINB)
 // Default mapping for small states (d <= 12), measured on B200:
 // about four particles per thread (P = m / 32 GW), one warp per sub-filter up
 // to m = 128, several sub-filters per CTA, at most ~80 registers (3 CTAs/SM).
@@ -59,9 +56,4 @@ extern const int kNumEntriesNJ28;
 #define PF_LATENCY_ENTRIES(NJ, RES)                                                                  \
   PF_ENTRY(NJ, 64, RES, 2, 4, 1, 1, 3), PF_ENTRY(NJ, 128, RES, 4, 2, 1, 1, 3),                      \
       PF_ENTRY(NJ, 256, RES, 8, 1, 1, 1, 3)
-#define PF_ENTRY_LARGE(NJ, M, RES, GW, S, NST, UNR, MINB)                                           \
-  {NJ, M, RES, GW, S, NST, UNR, MINB, 1,                                                             \
-   &StepKernel<KCfg<NJ, M, RES, GW, S, NST, UNR, MINB>>::prepare,                                    \
-   &StepKernel<KCfg<NJ, M, RES, GW, S, NST, UNR, MINB>>::launch,                                     \
-   &StepKernel<KCfg<NJ, M, RES, GW, S, NST, UNR, MINB>>::resample_debug,                             \
-   StepKernel<KCfg<NJ, M, RES, GW, S, NST, UNR, MINB>>::smem()}
+#define PF_ENTRY_LARGE(NJ, M, RES, GW, S, NST, UNR, MINB) PF_ENTRY_MT(ArmPlanar<NJ>, NJ, 1, M, RES, GW, S, NST, UNR, MINB)

@@ -42,19 +42,25 @@ Table tables(int i) {
   switch (i) {
     case 0: return {pf::kEntriesNJ2, pf::kNumEntriesNJ2};
     case 1: return {pf::kEntriesNJ5, pf::kNumEntriesNJ5};
-    default: return {pf::kEntriesNJ28, pf::kNumEntriesNJ28};
+    case 2: return {pf::kEntriesNJ28, pf::kNumEntriesNJ28};
+    default: return {pf::kEntriesLG1, pf::kNumEntriesLG1};
   }
 }
+constexpr int kTables = 4;
 
-// First entry matching (nj, m, res), or the PF_VARIANT-th one if set.
-const pf::KernelEntry* find_entry(int nj, int m, int res) {
+bool matches(const pf::KernelEntry& e, int model, int nj, int m, int res) {
+  return e.model == model && (model != PF_MODEL_ARM_PLANAR || e.nj == nj) && e.m == m && e.res == res;
+}
+
+// First entry matching (model, nj, m, res), or the PF_VARIANT-th one if set.
+const pf::KernelEntry* find_entry(int model, int nj, int m, int res) {
   const char* v = std::getenv("PF_VARIANT");
   int want = v ? std::atoi(v) : 0;
   const pf::KernelEntry* first = nullptr;
-  for (int ti = 0; ti < 3; ++ti) {
+  for (int ti = 0; ti < kTables; ++ti) {
     const Table t = tables(ti);
     for (int i = 0; i < t.n; ++i)
-      if (t.e[i].nj == nj && t.e[i].m == m && t.e[i].res == res) {
+      if (matches(t.e[i], model, nj, m, res)) {
         if (!first) first = &t.e[i];
         if (want-- == 0) return &t.e[i];
       }
@@ -64,11 +70,11 @@ const pf::KernelEntry* find_entry(int nj, int m, int res) {
 
 // Large shards take the entry flagged `large` when one is compiled.
 constexpr long long kLargeNLocal = 8192;
-const pf::KernelEntry* large_entry(int nj, int m, int res) {
-  for (int ti = 0; ti < 3; ++ti) {
+const pf::KernelEntry* large_entry(int model, int nj, int m, int res) {
+  for (int ti = 0; ti < kTables; ++ti) {
     const Table t = tables(ti);
     for (int i = 0; i < t.n; ++i)
-      if (t.e[i].nj == nj && t.e[i].m == m && t.e[i].res == res && t.e[i].large) return &t.e[i];
+      if (matches(t.e[i], model, nj, m, res) && t.e[i].large) return &t.e[i];
   }
   return nullptr;
 }
@@ -76,20 +82,21 @@ const pf::KernelEntry* large_entry(int nj, int m, int res) {
 // Small problems (too few sub-filters to keep the default mapping's groups
 // busy) are latency-bound: take the matching entry with the fewest particles
 // per thread.  PF_VARIANT, when set, wins.
-const pf::KernelEntry* latency_entry(int nj, int m, int res) {
+const pf::KernelEntry* latency_entry(int model, int nj, int m, int res) {
   const pf::KernelEntry* best = nullptr;
-  for (int ti = 0; ti < 3; ++ti) {
+  for (int ti = 0; ti < kTables; ++ti) {
     const Table t = tables(ti);
     for (int i = 0; i < t.n; ++i)
-      if (t.e[i].nj == nj && t.e[i].m == m && t.e[i].res == res &&
-          (!best || t.e[i].gw > best->gw))
+      if (matches(t.e[i], model, nj, m, res) && (!best || t.e[i].gw > best->gw))
         best = &t.e[i];
   }
   return best;
 }
 
 struct Geometry {
+  int model;          // pf_model_id
   int nj, d, m, deg, tt, E;
+  int zd, ud;         // measurement and control dimensions of the model
   long long N, R, C, n_local, g0, n_ext, M_local, ROW;
   bool central;   // one filter of m > 1024 particles, resampled globally (pf_central.cu)
   bool vose;      // resampler (central filter sizing)
@@ -98,10 +105,24 @@ struct Geometry {
 
 pf_status validate(const pf_config* cfg, const pf_model_params* mp, Geometry* g) {
   if (!cfg || !mp) return PF_EINVAL;
-  if (mp->model != PF_MODEL_ARM_PLANAR || mp->n_joints < 1) return PF_EINVAL;
-  if (!(mp->sigma_cam > 0.0f) || !(mp->sigma_theta_meas > 0.0f) || !(mp->sigma_theta >= 0.0f) ||
-      !(mp->sigma_pos >= 0.0f) || !(mp->sigma_vel >= 0.0f))
+  if (mp->model == PF_MODEL_ARM_PLANAR) {
+    if (mp->n_joints < 1) return PF_EINVAL;
+    if (!(mp->sigma_cam > 0.0f) || !(mp->sigma_theta_meas > 0.0f) || !(mp->sigma_theta >= 0.0f) ||
+        !(mp->sigma_pos >= 0.0f) || !(mp->sigma_vel >= 0.0f))
+      return PF_EINVAL;
+    g->model = PF_MODEL_ARM_PLANAR;
+    g->nj = mp->n_joints;
+    g->d = mp->n_joints + 4;
+    g->zd = mp->n_joints + 2;
+    g->ud = mp->n_joints;
+  } else if (mp->model == PF_MODEL_LINEAR_GAUSS_1D) {
+    if (!(mp->sigma_theta_meas > 0.0f) || !(mp->sigma_theta >= 0.0f)) return PF_EINVAL;
+    g->model = PF_MODEL_LINEAR_GAUSS_1D;
+    g->nj = 1;
+    g->d = g->zd = g->ud = 1;
+  } else {
     return PF_EINVAL;
+  }
   const int m = cfg->m;
   if (cfg->n_filters < 1 || cfg->t < 0 || cfg->world < 1 || cfg->rank < 0 || cfg->rank >= cfg->world)
     return PF_EINVAL;
@@ -118,9 +139,7 @@ pf_status validate(const pf_config* cfg, const pf_model_params* mp, Geometry* g)
     if (cfg->resampler == PF_RESAMPLE_VOSE && m > pf::kCentralVoseMax) return PF_EUNSUPPORTED;
     if (cfg->resample_policy != PF_POLICY_ALWAYS) return PF_EUNSUPPORTED;
     g->vose = cfg->resampler == PF_RESAMPLE_VOSE;
-    if (mp->n_joints != 2 && mp->n_joints != 5 && mp->n_joints != 28) return PF_EUNSUPPORTED;
-    g->nj = mp->n_joints;
-    g->d = mp->n_joints + 4;
+    if (g->model == PF_MODEL_ARM_PLANAR && g->nj != 2 && g->nj != 5 && g->nj != 28) return PF_EUNSUPPORTED;
     g->m = m;
     g->N = 1;
     g->deg = 0;
@@ -140,9 +159,7 @@ pf_status validate(const pf_config* cfg, const pf_model_params* mp, Geometry* g)
   if (cfg->topo != PF_TOPO_NONE && cfg->topo != PF_TOPO_RING && cfg->topo != PF_TOPO_TORUS2D &&
       cfg->topo != PF_TOPO_ALL2ALL)
     return PF_EINVAL;
-  if (!find_entry(mp->n_joints, m, cfg->resampler)) return PF_EUNSUPPORTED;
-  g->nj = mp->n_joints;
-  g->d = mp->n_joints + 4;
+  if (!find_entry(g->model, g->nj, m, cfg->resampler)) return PF_EUNSUPPORTED;
   g->m = m;
   g->N = cfg->n_filters;
   g->deg = cfg->topo == PF_TOPO_RING ? 2 : cfg->topo == PF_TOPO_TORUS2D ? 4 : cfg->topo == PF_TOPO_ALL2ALL ? 1 : 0;
@@ -186,7 +203,7 @@ struct pf_handle {
   pf_config cfg;
   pf_model_params mp;
   Geometry g;
-  pf::ArmConsts mc;
+  pf::ModelConsts mc;
   float* parts;      // [n_local][d+1][m] blocked SoA (row d = log-weight)
   float* mailbox;
   unsigned char* scratch;
@@ -202,6 +219,9 @@ struct pf_handle {
   // rank's peer block (flags + records), this rank's own block (cudaMalloc'd)
   bool peers;
   bool local_peers;   // connected by pf_peer_connect_local (one process, one device)
+  bool shared_device; // some connected peer runs on this rank's device (PDL off, see launch())
+  unsigned long long rv;          // peer rendezvous number of the last peer-mode launch
+  unsigned long long peer_timeout_ns;
   bool pdl;           // programmatic dependent launch of the step kernel (PF_NO_PDL unset at init)
   float* peer_mb[2];
   unsigned char* peer_blk[pf::kMaxRanks];
@@ -311,8 +331,8 @@ pf::StepParams base_params(pf_handle* h, long long k, int mode) {
 void host_inputs(pf_handle* h, pf::StepParams& p, const float* z, const float* u) {
   p.z = nullptr;
   p.u = nullptr;
-  std::memcpy(p.zin, z, sizeof(float) * (h->g.nj + 2));
-  std::memcpy(p.uin, u, sizeof(float) * h->g.nj);
+  std::memcpy(p.zin, z, sizeof(float) * h->g.zd);
+  std::memcpy(p.uin, u, sizeof(float) * h->g.ud);
 }
 
 // Centralized filter: particle buffers ping-pong ([2][D+1][M]), then the
@@ -369,20 +389,28 @@ pf::CentralParams central_params(pf_handle* h, long long k) {
   return c;
 }
 
-pf_status launch(pf_handle* h, const pf::StepParams& p) {
-  // programmatic dependent launch, except for shards of one process sharing a
-  // device through the peer transport (a next step's waiting CTAs could hold
-  // the SMs another shard's current step needs to reach the rendezvous)
-  return sticky(h, h->ke->launch(p, h->grid, h->stream, h->pdl && !h->local_peers));
+pf_status launch(pf_handle* h, const pf::StepParams& p0) {
+  pf::StepParams p = p0;
+  if (h->peers && (p.mode == pf::MODE_STEP || p.mode == pf::MODE_PUBLISH)) {
+    // every rank makes the same sequence of peer-mode launches (steps and
+    // publishes are collective), so the rendezvous numbers agree
+    p.rv = ++h->rv;
+    p.peer_timeout_ns = h->peer_timeout_ns;
+  }
+  // programmatic dependent launch, except when a connected peer shares this
+  // device (shards of one process, or processes on one GPU): a next step's
+  // waiting CTAs could hold the SMs another shard's current step needs to
+  // reach the rendezvous
+  return sticky(h, h->ke->launch(p, h->grid, h->stream, h->pdl && !h->local_peers && !h->shared_device));
 }
 pf_status launch_central(pf_handle* h, const pf::CentralParams& c) {
-  return sticky(h, pf::central_step(h->g.nj, c, h->grid, h->stream));
+  return sticky(h, pf::central_step(h->g.model, h->g.nj, c, h->grid, h->stream));
 }
 void host_inputs(pf_handle* h, pf::CentralParams& c, const float* z, const float* u) {
   c.z = nullptr;
   c.u = nullptr;
-  std::memcpy(c.zin, z, sizeof(float) * (h->g.nj + 2));
-  std::memcpy(c.uin, u, sizeof(float) * h->g.nj);
+  std::memcpy(c.zin, z, sizeof(float) * h->g.zd);
+  std::memcpy(c.uin, u, sizeof(float) * h->g.ud);
 }
 
 __global__ void pf_init_kernel(float* parts, int m, long long M_local, uint32_t p0, int d, const float* mu0,
@@ -506,27 +534,28 @@ pf_status pf_init(const pf_config* cfg, const pf_model_params* model, const pf_b
   h->cfg = *cfg;
   h->mp = *model;
   h->g = g;
-  // F9/F10 model constants: fp32 operations, exactly as the contract states
-  h->mc.lj = model->arm_length / static_cast<float>(model->n_joints);
+  // F8-F10 model constants: fp32 operations, exactly as the contract states
+  // (pf_model.cuh: the 1-D linear-Gaussian model reads hs, s_th, inv_thm)
+  h->mc.lj = g.model == PF_MODEL_ARM_PLANAR ? model->arm_length / static_cast<float>(model->n_joints) : 0.0f;
   h->mc.hs = model->h_s;
   h->mc.s_th = model->sigma_theta;
   h->mc.s_pos = model->sigma_pos;
   h->mc.s_vel = model->sigma_vel;
-  h->mc.inv_cam = 1.0f / model->sigma_cam;
+  h->mc.inv_cam = g.model == PF_MODEL_ARM_PLANAR ? 1.0f / model->sigma_cam : 0.0f;
   h->mc.inv_thm = 1.0f / model->sigma_theta_meas;
   h->parts = static_cast<float*>(buffers->state);
   h->mailbox = static_cast<float*>(buffers->mailbox);
   h->scratch = static_cast<unsigned char*>(buffers->scratch);
   h->stream = static_cast<cudaStream_t>(cuda_stream);
   h->step = 0;
-  h->ke = g.central ? nullptr : find_entry(g.nj, g.m, cfg->resampler);
+  h->ke = g.central ? nullptr : find_entry(g.model, g.nj, g.m, cfg->resampler);
   h->err = PF_OK;
   int dev = 0, sms = 0, bps = 0;
   cudaError_t e = cudaGetDevice(&dev);
   if (e == cudaSuccess) e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
   if (e == cudaSuccess && g.central) {
     bps = 1;
-    h->grid = pf::central_grid(g.nj, sms);
+    h->grid = pf::central_grid(g.model, g.nj, sms);
     if (h->grid < 1) e = cudaErrorInvalidConfiguration;
   } else if (e == cudaSuccess) {
     e = h->ke->prepare(&bps);
@@ -537,6 +566,9 @@ pf_status pf_init(const pf_config* cfg, const pf_model_params* model, const pf_b
   if (e == cudaSuccess) e = cudaHostGetDevicePointer(reinterpret_cast<void**>(&h->rec_host_dev), h->rec_host, 0);
   if (e == cudaSuccess) {
     h->mapped = std::getenv("PF_NO_MAPPED") == nullptr;
+    const char* to = std::getenv("PF_PEER_TIMEOUT_MS");
+    const long long ms = to ? std::atoll(to) : 30000;
+    h->peer_timeout_ns = static_cast<unsigned long long>(ms > 0 ? ms : 30000) * 1000000ull;
     h->pdl = std::getenv("PF_NO_PDL") == nullptr;
     h->last_mapped = false;
     reinterpret_cast<volatile uint32_t*>(h->rec_host)[pf::kRecordSeq] = 0xFFFFFFFFu;
@@ -546,7 +578,7 @@ pf_status pf_init(const pf_config* cfg, const pf_model_params* model, const pf_b
     return PF_ECUDA;
   }
   if (!g.central && !std::getenv("PF_VARIANT") && g.n_local >= kLargeNLocal) {
-    const pf::KernelEntry* le = large_entry(g.nj, g.m, cfg->resampler);
+    const pf::KernelEntry* le = large_entry(g.model, g.nj, g.m, cfg->resampler);
     if (le && le != h->ke) {
       int b2 = 0;
       if (le->prepare(&b2) == cudaSuccess && b2 >= 1) {
@@ -558,7 +590,7 @@ pf_status pf_init(const pf_config* cfg, const pf_model_params* model, const pf_b
   // fewer sub-filters than a quarter of the default mapping's groups: switch
   // to the lowest-latency mapping (more threads per sub-filter)
   if (!g.central && !std::getenv("PF_VARIANT") && g.n_local * 4 <= static_cast<long long>(bps) * sms * h->ke->s) {
-    const pf::KernelEntry* le = latency_entry(g.nj, g.m, cfg->resampler);
+    const pf::KernelEntry* le = latency_entry(g.model, g.nj, g.m, cfg->resampler);
     if (le && le != h->ke) {
       int b2 = 0;
       if (le->prepare(&b2) == cudaSuccess && b2 >= 1) {
@@ -643,14 +675,14 @@ pf_status pf_step_batch(pf_handle* h, int32_t T, const float* zs, const float* u
   if (!h || T < 0 || (T > 0 && (!zs || !us))) return PF_EINVAL;
   if (h->err != PF_OK) return h->err;
   if (h->cfg.world != 1) return PF_ESTATE;
-  const int nj = h->g.nj;
+  const int zd = h->g.zd, ud = h->g.ud;
   h->last_mapped = false;
   for (int32_t s = 0; s < T; ++s) {
     const long long k = h->step + 1;
     if (h->g.central) {
       pf::CentralParams c = central_params(h, k);
-      c.z = zs + static_cast<long long>(s) * (nj + 2);
-      c.u = us + static_cast<long long>(s) * nj;
+      c.z = zs + static_cast<long long>(s) * zd;
+      c.u = us + static_cast<long long>(s) * ud;
       c.est_out = est ? est + static_cast<long long>(s) * (4 + h->g.d) : nullptr;
       c.record_host = nullptr;   // device-resident pipeline: records stay on the device
       const pf_status st = launch_central(h, c);
@@ -659,8 +691,8 @@ pf_status pf_step_batch(pf_handle* h, int32_t T, const float* zs, const float* u
       continue;
     }
     pf::StepParams p = base_params(h, k, pf::MODE_STEP);
-    p.z = zs + static_cast<long long>(s) * (nj + 2);
-    p.u = us + static_cast<long long>(s) * nj;
+    p.z = zs + static_cast<long long>(s) * zd;
+    p.u = us + static_cast<long long>(s) * ud;
     p.est_out = est ? est + static_cast<long long>(s) * (4 + h->g.d) : nullptr;
     p.record_host = nullptr;   // device-resident pipeline: records stay on the device
     if (h->trace) {
@@ -687,8 +719,10 @@ pf_status pf_estimate(pf_handle* h, float* x_hat, float* logw, int64_t* idx) {
   cudaError_t e = cudaSuccess;
   if (h->last_mapped) {
     const uint32_t want = static_cast<uint32_t>(h->step);
-    volatile const uint32_t* seq = reinterpret_cast<volatile const uint32_t*>(h->rec_host + pf::kRecordSeq);
-    for (unsigned it = 1; *seq != want; ++it) {
+    // acquire: the record loads below may not be reordered before the step
+    // number (the kernel wrote the record first, then a system-scope fence)
+    const uint32_t* seq = reinterpret_cast<const uint32_t*>(h->rec_host + pf::kRecordSeq);
+    for (unsigned it = 1; __atomic_load_n(seq, __ATOMIC_ACQUIRE) != want; ++it) {
       if ((it & 1023u) == 0u) {
         e = cudaStreamQuery(h->stream);
         if (e != cudaErrorNotReady) break;
@@ -706,8 +740,13 @@ pf_status pf_estimate(pf_handle* h, float* x_hat, float* logw, int64_t* idx) {
   }
   float rec[4 + 32 + 4];
   std::memcpy(rec, const_cast<const float*>(h->rec_host), sizeof(float) * (4 + h->g.d));
-  uint32_t lo;
+  uint32_t lo, status;
   std::memcpy(&lo, &rec[0], 4);
+  std::memcpy(&status, &rec[3], 4);
+  if (status == pf::kStatusPeerTimeout) {   // the device rendezvous gave up on a rank (sticky)
+    if (h->err == PF_OK) h->err = PF_ETIMEOUT;
+    return PF_ETIMEOUT;
+  }
   std::memcpy(x_hat, rec + 4, sizeof(float) * h->g.d);
   if (logw) *logw = rec[2];
   if (idx) *idx = static_cast<int64_t>(0xFFFFFFFFu - lo);
@@ -972,10 +1011,9 @@ pf_status pf_get_trace(pf_handle* h, int64_t* src, int32_t* ancestors) {
 
 // ---- peer transport (NVLink / NVSwitch peer memory via CUDA IPC) ----------
 namespace {
-// [kMaxRanks] u64 flags + [kMaxRanks][kPeerRec] record floats + [kMaxRanks][kPeerPool] pool floats
-constexpr size_t kPeerBlockBytes = 40960;
-static_assert(sizeof(u64) * pf::kMaxRanks + sizeof(float) * pf::kMaxRanks * (pf::kPeerRec + pf::kPeerPool) <=
-                  kPeerBlockBytes, "");
+// [kMaxRanks] u64 flags + [2][kMaxRanks][kPeerRec] record floats + [2][kMaxRanks][kPeerPool] pool floats
+constexpr size_t kPeerBlockBytes = 81920;
+static_assert(pf::kPeerBlockUsed <= kPeerBlockBytes, "peer block");
 
 pf_status peer_check(const pf_handle* h) {
   if (!h) return PF_EINVAL;
@@ -1030,6 +1068,11 @@ pf_status pf_peer_export(pf_handle* h, uint8_t* blob) {
   std::memcpy(blob + 72, &hb, sizeof(hb));
   const int64_t rank = h->cfg.rank;
   std::memcpy(blob + 136, &rank, sizeof(rank));
+  // the device's PCI bus id (peers on the same device turn PDL off)
+  int dev = 0;
+  e = cudaGetDevice(&dev);
+  if (e == cudaSuccess) e = cudaDeviceGetPCIBusId(reinterpret_cast<char*>(blob + 144), 16, dev);
+  if (e != cudaSuccess) return sticky(h, e);
   return PF_OK;
 }
 
@@ -1041,11 +1084,14 @@ pf_status pf_peer_connect(pf_handle* h, const uint8_t* blobs) {
   const int prev = (r + W - 1) % W, next = (r + 1) % W;
   unsigned char* blks[pf::kMaxRanks] = {};
   float* mbs[pf::kMaxRanks] = {};
+  const uint8_t* mine = blobs + static_cast<size_t>(r) * PF_PEER_BLOB_BYTES;
+  bool shared = false;
   for (int q = 0; q < W; ++q) {
     const uint8_t* b = blobs + static_cast<size_t>(q) * PF_PEER_BLOB_BYTES;
     int64_t qr;
     std::memcpy(&qr, b + 136, sizeof(qr));
     if (qr != q) return PF_EINVAL;
+    if (q != r && std::memcmp(b + 144, mine + 144, 16) == 0) shared = true;
     if (q == r) {
       blks[q] = h->own_blk;
       mbs[q] = h->mailbox;
@@ -1071,6 +1117,7 @@ pf_status pf_peer_connect(pf_handle* h, const uint8_t* blobs) {
     }
   }
   set_peers(h, mbs[prev], mbs[next], blks);
+  h->shared_device = shared;
   return PF_OK;
 }
 
@@ -1114,7 +1161,8 @@ const char* pf_strerror(pf_status s) {
     case PF_ENOMEM: return "host allocation failed";
     case PF_ECUDA: return "CUDA error";
     case PF_ESTATE: return "call not valid in the handle's state";
-    case PF_EUNSUPPORTED: return "configuration not compiled (n_joints, m)";
+    case PF_EUNSUPPORTED: return "configuration not compiled (model, n_joints, m)";
+    case PF_ETIMEOUT: return "peer rendezvous timed out (a rank did not arrive)";
     default: return "unknown pf_status";
   }
 }
@@ -1123,9 +1171,10 @@ pf_status pf_last_error(const pf_handle* h) { return h ? h->err : PF_EINVAL; }
 
 int32_t pf_supported(int32_t* n_joints, int32_t* m, int32_t cap) {
   int32_t n = 0;
-  for (int ti = 0; ti < 3; ++ti) {
+  for (int ti = 0; ti < kTables; ++ti) {
     const Table t = tables(ti);
     for (int i = 0; i < t.n; ++i) {
+      if (t.e[i].model != PF_MODEL_ARM_PLANAR) continue;
       bool dup = false;
       for (int j = 0; j < i; ++j) dup = dup || (t.e[j].m == t.e[i].m && t.e[j].nj == t.e[i].nj);
       if (t.e[i].res != 0 || dup) continue;

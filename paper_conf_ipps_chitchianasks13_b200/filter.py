@@ -38,6 +38,33 @@ class ArmModel:
                                  self.sigma_pos, self.sigma_vel, self.sigma_cam, self.sigma_theta_meas)
 
 
+@dataclass
+class LinearGaussModel:
+    """1-D linear-Gaussian model (pf.h PF_MODEL_LINEAR_GAUSS_1D; pf_model.cuh):
+    theta_k = theta_{k-1} + h_s u + w, w ~ N(0, sigma_theta^2); z = theta + v,
+    v ~ N(0, sigma_theta_meas^2) — one joint of the arm with its angle sensor,
+    the Kalman special case of SURVEY §8(c)."""
+    h_s: float = 0.1
+    sigma_theta: float = 0.1
+    sigma_theta_meas: float = 0.1
+    n_joints: int = 1
+
+    @property
+    def d(self) -> int:
+        return 1
+
+    def c(self) -> B.pf_model_params:
+        return B.pf_model_params(B.PF_MODEL_LINEAR_GAUSS_1D, 1, 0.0, self.h_s, self.sigma_theta, 0.0, 0.0, 0.0,
+                                 self.sigma_theta_meas)
+
+
+def _dims(model) -> tuple[int, int]:
+    """(measurement, control) dimensions of a model."""
+    if isinstance(model, LinearGaussModel):
+        return 1, 1
+    return model.n_joints + 2, model.n_joints
+
+
 POLICY = {"always": B.PF_POLICY_ALWAYS, "ess": B.PF_POLICY_ESS, "freq": B.PF_POLICY_FREQ}
 
 
@@ -73,7 +100,7 @@ class ParticleFilter:
     probability ``policy_value`` per step).
     """
 
-    def __init__(self, mu0, sigma0, model: ArmModel | None = None, m: int = 256, n_filters: int = 4096,
+    def __init__(self, mu0, sigma0, model: ArmModel | LinearGaussModel | None = None, m: int = 256, n_filters: int = 4096,
                  t: int = 1, topo: str = "ring", resampler: str = "rws", seed: int = 0, rank: int = 0,
                  world: int = 1, torus_rows: int = 0, torus_cols: int = 0, device_inputs: bool = False,
                  device: torch.device | int | None = None, stream: torch.cuda.Stream | None = None,
@@ -106,8 +133,9 @@ class ParticleFilter:
         # per-step host path (e2e): persistent input / output buffers with
         # their pointers taken once (numpy pointer extraction costs ~1 us)
         self._device_inputs = bool(self.cfg.flags & B.PF_DEVICE_INPUTS)
-        self._zin = np.zeros(self.nj + 2, np.float32)
-        self._uin = np.zeros(self.nj, np.float32)
+        self.zd, self.ud = _dims(self.model)
+        self._zin = np.zeros(self.zd, np.float32)
+        self._uin = np.zeros(self.ud, np.float32)
         self._zin_p, self._uin_p, self._xhat_p = self._zin.ctypes.data, self._uin.ctypes.data, self._xhat.ctypes.data
         self._step_fn, self._est_fn = B.lib().pf_step, B.lib().pf_estimate
         self._lw, self._idx = B.C.c_float(), B.C.c_int64()
@@ -148,7 +176,7 @@ class ParticleFilter:
         self._k += 1
 
     def step_batch(self, zs: torch.Tensor, us: torch.Tensor, est: torch.Tensor | None = None) -> None:
-        """T steps with device-resident inputs zs [T][nj+2], us [T][nj]; est [T][4+d]."""
+        """T steps with device-resident inputs zs [T][zd], us [T][ud]; est [T][4+d]."""
         assert zs.is_cuda and us.is_cuda and zs.dtype == torch.float32 and us.dtype == torch.float32
         B.pf_step_batch(self.h, zs.shape[0], zs.data_ptr(), us.data_ptr(), None if est is None else est.data_ptr())
         self._k += zs.shape[0]

@@ -99,3 +99,22 @@ def random_q(N: int, m: int, seed: int, kind: str = "mixed") -> np.ndarray:
         ell[rng.random((N, m)) < 0.2] = -30.0
         q = np.floor(np.exp(ell - ell.max(1, keepdims=True)) * (1 << 22)).astype(np.uint32)
     return q
+
+
+def make_lg_trajectory(T: int, seed: int = 0, h_s: float = 0.1, sigma_theta: float = 0.1,
+                       sigma_meas: float = 0.1, prior_offset: float = 0.2, prior_std: float = 0.25) -> dict:
+    """The 1-D linear-Gaussian plant (pf_model.cuh LinearGauss1D: one joint with
+    its angle sensor): theta_k = theta_{k-1} + h_s u_{k-1} + sigma_theta xi,
+    z_k = theta_k + sigma_meas xi, u_k = 0.5 sin(2 pi k / T).  Arrays shaped
+    like make_trajectory's with d = zd = ud = 1: X[T+1, 1], Z[T+1, 1] (Z[0]
+    unused), U[T+1, 1]; prior mu0 = theta_0 + prior_offset, sigma0 = prior_std."""
+    rng = np.random.default_rng(50000 + seed)
+    U = 0.5 * np.sin(2 * np.pi * np.arange(T + 1) / T)[:, None]
+    theta = np.zeros((T + 1, 1))
+    theta[0] = 0.3
+    for t in range(1, T + 1):
+        theta[t] = theta[t - 1] + h_s * U[t - 1] + sigma_theta * rng.standard_normal(1)
+    Z = theta + sigma_meas * rng.standard_normal((T + 1, 1))
+    f = lambda a: np.ascontiguousarray(a, np.float32)
+    return {"X": f(theta), "Z": f(Z), "U": f(U), "mu0": f(theta[0] + prior_offset),
+            "sigma0": f(np.full(1, prior_std)), "T": T, "n_joints": 1, "d": 1}

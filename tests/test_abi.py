@@ -88,3 +88,19 @@ def test_unsupported_model(B):
     assert B.lib().pf_query_sizes(C.byref(_cfg(B)), C.byref(_model(B, 7)), C.byref(out)) == B.PF_EUNSUPPORTED
     assert (5, 256) in B.pf_supported() and (28, 256) in B.pf_supported()
     assert B.pf_strerror(B.PF_EINVAL).startswith("invalid")
+
+
+def test_model_selection(B):
+    # the model id selects the compiled model instance (pf.h pf_model_id)
+    lg = B.pf_model_params(B.PF_MODEL_LINEAR_GAUSS_1D, 0, 0.0, 0.1, 0.1, 0.0, 0.0, 0.0, 0.2)
+    s = B.pf_query_sizes(_cfg(B, m=256, n_filters=8), lg)
+    assert s.state == 4 * (1 + 1) * 256 * 8                 # d = 1: one state row + the log-weight row
+    assert s.mailbox == 4 * 2 * 8 * 1 * (1 + 2)
+    out = B.pf_sizes()
+    # centralized linear-Gaussian filter (m = 10^5-class, a multiple of 4096)
+    assert B.lib().pf_query_sizes(C.byref(_cfg(B, m=102400, n_filters=1, t=0, topo=0)), C.byref(lg),
+                                  C.byref(out)) == B.PF_OK
+    bad = B.pf_model_params(7, 5, 1.0, 0.1, 0.1, 0.1, 0.1, 0.1, 0.1)
+    assert B.lib().pf_query_sizes(C.byref(_cfg(B)), C.byref(bad), C.byref(out)) == B.PF_EINVAL
+    lg_bad = B.pf_model_params(B.PF_MODEL_LINEAR_GAUSS_1D, 0, 0.0, 0.1, 0.1, 0.0, 0.0, 0.0, 0.0)   # sigma_meas = 0
+    assert B.lib().pf_query_sizes(C.byref(_cfg(B)), C.byref(lg_bad), C.byref(out)) == B.PF_EINVAL

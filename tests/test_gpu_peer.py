@@ -115,3 +115,69 @@ def test_peer_transport_two_processes_ipc(P, topo, tmp_path):
     for r, (p, out) in enumerate(zip(procs, outs)):
         assert p.returncode == 0, f"rank {r}:\n{out[-3000:]}"
         assert f"rank {r} ok" in out
+
+
+@pytest.mark.timeout(120)
+@pytest.mark.parametrize("topo,t", [("ring", 1), ("all2all", 2)])
+def test_peer_back_to_back_skewed(P, orc, W, topo, t):
+    # steps launched back to back with NO host synchronization between them,
+    # one shard's stream delayed by a sleep before every other step, each
+    # step's record captured on the device: every step's estimate must still
+    # equal the oracle's (double-buffered records / pool rows)
+    import torch
+    nj, m, N, world, T = 5, 64, 16, 2, 10
+    tr = W.make_trajectory(nj, T, 2)
+    kw = dict(m=m, n_filters=N, t=t, topo=topo, resampler="rws", seed=17)
+    shards = [P.ParticleFilter(tr["mu0"], tr["sigma0"], P.ArmModel(n_joints=nj), rank=r, world=world,
+                               stream=torch.cuda.Stream(), **kw) for r in range(world)]
+    P.ParticleFilter.peer_connect_local(shards)
+    # load the sleep kernel's module now: a lazily loaded module can only be
+    # loaded between kernels, so loading it while rank 0's step kernel waits
+    # at the rendezvous would stall the one host thread that must launch
+    # rank 1's step (caught by the rendezvous timeout, PF_ETIMEOUT)
+    torch.cuda._sleep(1)
+    torch.cuda.synchronize()
+    recs = [[] for _ in shards]
+    for k in range(1, T + 1):
+        for r, s in enumerate(shards):
+            if r == 1 and k % 2 == 0:
+                with torch.cuda.stream(s.stream):
+                    torch.cuda._sleep(2_000_000)      # ~1 ms: rank 1 reaches the rendezvous late
+            s.step(tr["Z"][k], tr["U"][k - 1])
+            with torch.cuda.stream(s.stream):
+                recs[r].append(s.record.clone())
+    torch.cuda.synchronize()
+    o = orc.Filter(orc.Config(**kw), orc.Model(n_joints=nj), tr["mu0"], tr["sigma0"])
+    for k in range(1, T + 1):
+        o.step(tr["Z"][k], tr["U"][k - 1])
+        xo, lo, io = o.estimate()
+        for r in range(world):
+            rec = recs[r][k - 1].cpu().numpy()
+            idx = 0xFFFFFFFF - int(rec[:1].view(np.uint32)[0])
+            assert idx == io, (r, k, idx, io)
+            assert rec[3:4].view(np.uint32)[0] == 0          # status ok
+            np.testing.assert_array_equal(rec[4:4 + nj + 4], xo)
+    for s in shards:
+        s.close()
+
+
+@pytest.mark.timeout(120)
+def test_peer_rendezvous_timeout_is_reported(P, W, monkeypatch):
+    # a rank that never arrives: the waiting rank's kernel gives up after
+    # PF_PEER_TIMEOUT_MS and pf_estimate returns PF_ETIMEOUT (sticky) — the
+    # GPU does not hang
+    import torch
+    monkeypatch.setenv("PF_PEER_TIMEOUT_MS", "300")
+    nj = 2
+    tr = W.make_trajectory(nj, 4, 0)
+    kw = dict(m=64, n_filters=4, t=1, topo="ring", seed=1)
+    shards = [P.ParticleFilter(tr["mu0"], tr["sigma0"], P.ArmModel(n_joints=nj), rank=r, world=2,
+                               stream=torch.cuda.Stream(), **kw) for r in range(2)]
+    P.ParticleFilter.peer_connect_local(shards)
+    shards[0].step(tr["Z"][1], tr["U"][0])          # rank 1 never steps
+    with pytest.raises(P.B.PFError, match="timed out"):
+        shards[0].estimate()
+    with pytest.raises(P.B.PFError):                # sticky
+        shards[0].step(tr["Z"][2], tr["U"][1])
+    for s in shards:
+        s.close()
