@@ -471,6 +471,9 @@ __device__ __forceinline__ void resample_group(const uint32_t (&q)[C::P], const 
       const u64 slot1 = static_cast<u64>(C::slot(G.t, j)) + 1;
       Einc = Dinc + static_cast<u64>(M) * qinc[j] - slot1 * Qg;
     };
+    // Lists: small slots ascending with their EXCLUSIVE deficit sums A_i =
+    // D_{i-1} (A_0 = 0) at [0, nL), large slots ascending with their
+    // inclusive excess sums E_j at [nL, M) (both sequences sorted).
 #pragma unroll
     for (int j = 0; j < P; ++j) {
       bool small;
@@ -480,54 +483,64 @@ __device__ __forceinline__ void resample_group(const uint32_t (&q)[C::P], const 
       const int s = C::slot(G.t, j);
       if (small) {
         S.lists[ls] = s;
-        S.scan[ls] = Dinc;
+        S.scan[ls] = Dinc - (Qg - a);
       } else {
         S.lists[nL + (s - ls)] = s;
         S.scan[nL + (s - ls)] = Einc;
       }
     }
     gsync<C::GW>(G.g);
+    // The closed form of the sweep (R10) is a MERGE of the sorted sequences
+    // A (small) and E (large) with "A first on ties":
+    //   small L[i]: alias = H[lower_bound(E, A_i)] = H[#E before A_i],
+    //               prob = a = Q - (A_{i+1} - A_i)   (A_nL := D_last);
+    //   large H[j] with E_j < D_last: prob = Q + E_j - D[upper_bound(D, E_j)]
+    //               = Q + E_j - (the next A after E_j in merge order, or D_last),
+    //               alias = H[j + 1]; otherwise prob = Q, alias = itself.
+    // Merge path: thread t emits merged positions [tP, tP + P) after ONE
+    // binary search for its split on the diagonal (instead of one search per
+    // slot), then P sequential merge steps.
+    {
+      const int nH = M - nL;
+      const int diag = G.t * P;
+      int lo = diag - nH > 0 ? diag - nH : 0, hi = diag < nL ? diag : nL;
+      while (lo < hi) {   // first i with A_i > E_{diag-1-i} (A before E on ties)
+        const int mid = (lo + hi) >> 1;
+        if (S.scan[mid] <= S.scan[nL + diag - 1 - mid]) lo = mid + 1;
+        else hi = mid;
+      }
+      int i = lo, jj = diag - lo;
+      u64 Ai = i < nL ? S.scan[i] : Dtot;        // head of A (D_last past the end)
+      u64 Bj = jj < nH ? S.scan[nL + jj] : ~0ull;
 #pragma unroll
-    for (int j = 0; j < P; ++j) {
-      bool small;
-      u64 a, Dinc, Einc;
-      int ls;
-      cls(j, small, a, Dinc, Einc, ls);
-      const int s = C::slot(G.t, j);
-      // one branch-free search per slot, the same for small and large slots
-      // (no divergence between them): small -> first E over H that is >=
-      // D_{i-1}; large with E < D_last -> first D over L that is > E, i.e.
-      // >= E + 1 (integers).  log2(M) predicated halving steps.
-      const bool srch = small || Einc < Dtot;
-      const u64 key = small ? Dinc - (Qg - a) : Einc + 1;
-      int base = small ? nL : 0;
-      int len = !srch ? 1 : (small ? M - nL : nL);
-#pragma unroll
-      for (int it = 1; it < M; it <<= 1) {
-        if (len > 1) {
-          const int half = len >> 1;
-          if (S.scan[base + half] < key) base += half;
-          len -= half;
+      for (int e = 0; e < P; ++e) {
+        int s, al;
+        u64 pr;
+        if (i < nL && Ai <= Bj) {   // small slot L[i]
+          s = S.lists[i];
+          const u64 An = i + 1 < nL ? S.scan[i + 1] : Dtot;
+          pr = Qg - (An - Ai);
+          al = S.lists[nL + jj];
+          ++i;
+          Ai = An;
+        } else {                    // large slot H[jj]
+          s = S.lists[nL + jj];
+          if (Bj < Dtot) {
+            pr = Qg + Bj - Ai;
+            al = S.lists[nL + jj + 1];
+          } else {
+            pr = Qg;
+            al = s;
+          }
+          ++jj;
+          Bj = jj < nH ? S.scan[nL + jj] : ~0ull;
         }
-      }
-      const int pos = base + (srch && S.scan[base] < key ? 1 : 0);   // absolute index in scan / lists
-      u64 pr;
-      int al;
-      if (small) {
-        pr = a;
-        al = S.lists[pos];
-      } else if (srch) {
-        pr = Qg + Einc - S.scan[pos];
-        al = S.lists[nL + (s - ls) + 1];
-      } else {
-        pr = Qg;
-        al = s;
-      }
-      S.prob[s] = pr;
-      S.alias[s] = al;
-      if (prob_out) {
-        prob_out[s] = pr;
-        alias_out[s] = al;
+        S.prob[s] = pr;
+        S.alias[s] = al;
+        if (prob_out) {
+          prob_out[s] = pr;
+          alias_out[s] = al;
+        }
       }
     }
     const u64 Q2 = Qg;
