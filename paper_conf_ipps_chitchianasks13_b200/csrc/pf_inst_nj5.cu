@@ -9,7 +9,7 @@ const KernelEntry kEntriesNJ5[] = {
     PF_SMALL_D_ENTRIES(5, 0), PF_SMALL_D_ENTRIES(5, 1),
     PF_LATENCY_ENTRIES(5, 0), PF_LATENCY_ENTRIES(5, 1),
     // measured best for large shards (C5: 16M particles per GPU)
-    PF_ENTRY_LARGE(5, 256, 0, 2, 4, 1, 1, 4), PF_ENTRY_LARGE(5, 256, 1, 2, 3, 1, 1, 4),
+    PF_ENTRY_LARGE(5, 256, 0, 2, 4, 1, 1, 4), PF_ENTRY_LARGE(5, 256, 1, 2, 7, 1, 1, 2),
     PF_ENTRY_LARGE(5, 512, 0, 4, 1, 1, 1, 3),
     // alternatives for PF_VARIANT tuning of configs C2 / C5 (m = 256)
     PF_ENTRY(5, 256, 0, 8, 1, 2, 1, 4), PF_ENTRY(5, 256, 0, 1, 8, 1, 1, 3), PF_ENTRY(5, 256, 0, 4, 2, 1, 1, 3),
@@ -19,6 +19,8 @@ const KernelEntry kEntriesNJ5[] = {
     PF_ENTRY(5, 256, 0, 2, 3, 1, 4, 3),
     PF_ENTRY(5, 256, 1, 2, 4, 1, 1, 4), PF_ENTRY(5, 256, 1, 2, 3, 1, 1, 4),
     PF_ENTRY(5, 256, 0, 2, 3, 2, 1, 3), PF_ENTRY(5, 256, 0, 2, 4, 2, 1, 2), PF_ENTRY(5, 256, 0, 2, 2, 2, 1, 4),
+    // Vose with the round-2 table footprint (RWS + 2 KB per group): 14 groups per SM
+    PF_ENTRY(5, 256, 1, 2, 2, 1, 1, 7), PF_ENTRY(5, 256, 1, 1, 7, 1, 1, 2),
 };
 const int kNumEntriesNJ5 = sizeof(kEntriesNJ5) / sizeof(kEntriesNJ5[0]);
 }  // namespace pf

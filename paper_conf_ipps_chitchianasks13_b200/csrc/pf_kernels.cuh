@@ -195,10 +195,13 @@ struct KCfg {
   static constexpr size_t g_stage = 0;
   static constexpr size_t g_scan = NSTAGE * stage_bytes;                          // u64 [M]; after the
                                                                                   // resample: Philox words
+  // Vose: the second scan, then the alias table: prob u32 [M] + alias u16 [M]
+  // when Q <= M 2^22 fits 32 bits (m <= 512), else prob u64 [M] + alias int [M]
+  // (the small/large lists live in the stage's log-weight row, free by then)
+  static constexpr bool PROB32 = (RES == RES_VOSE) && M <= 512;
   static constexpr size_t g_prob = g_scan + sizeof(u64) * M;                      // u64 [M]  (Vose)
-  static constexpr size_t g_alias = g_prob + (RES == RES_VOSE ? sizeof(u64) * M : 0);
-  static constexpr size_t g_lists = g_alias + (RES == RES_VOSE ? sizeof(int) * M : 0);
-  static constexpr size_t g_red = g_lists + (RES == RES_VOSE ? sizeof(int) * M : 0);   // u64 [2][32]
+  static constexpr size_t g_alias = g_prob + (RES == RES_VOSE ? sizeof(u64) * M : 0);   // int [M] (!PROB32)
+  static constexpr size_t g_red = g_alias + ((RES == RES_VOSE && !PROB32) ? sizeof(int) * M : 0);   // u64 [2][32]
   static constexpr size_t g_cand = g_red + sizeof(u64) * 64;                     // u64 [GW KMAX + GW]
   static constexpr size_t g_misc = g_cand + sizeof(u64) * GW * (KMAX + 1);       // int [GW][2][KMAX]
   static constexpr size_t g_bar = g_misc + sizeof(int) * GW * 2 * KMAX;          // u64 [2] + next [2]
@@ -381,10 +384,10 @@ __device__ __forceinline__ void search_levels(uint32_t& a, uint32_t c) {
 
 // ---------------------------------------------------------- resampling
 struct ResampleSmem {
-  u64* scan;    // [M] RWS: inclusive sums C (u32 or u64); Vose: D over L, then E over H
-  u64* prob;    // [M] Vose
-  int* alias;   // [M] Vose
-  int* lists;   // [M] Vose: L ascending then H ascending
+  u64* scan;    // [M] RWS: inclusive sums C (u32 or u64); Vose: exclusive D over L, then E over H
+  u64* prob;    // [M] Vose: the second scan, then the table (KCfg::PROB32: u32 prob [M] + u16 alias [M])
+  int* alias;   // [M] Vose, !PROB32
+  int* lists;   // [M] Vose: L ascending then H ascending (the stage's log-weight row)
 };
 
 // Ancestors anc[P] of the thread's slots (a8) from integer weights q[P]
@@ -535,8 +538,13 @@ __device__ __forceinline__ void resample_group(const uint32_t (&q)[C::P], const 
           ++jj;
           Bj = jj < nH ? S.scan[nL + jj] : ~0ull;
         }
-        S.prob[s] = pr;
-        S.alias[s] = al;
+        if constexpr (C::PROB32) {
+          reinterpret_cast<uint32_t*>(S.prob)[s] = static_cast<uint32_t>(pr);
+          reinterpret_cast<uint16_t*>(reinterpret_cast<uint32_t*>(S.prob) + M)[s] = static_cast<uint16_t>(al);
+        } else {
+          S.prob[s] = pr;
+          S.alias[s] = al;
+        }
         if (prob_out) {
           prob_out[s] = pr;
           alias_out[s] = al;
@@ -549,7 +557,12 @@ __device__ __forceinline__ void resample_group(const uint32_t (&q)[C::P], const 
     for (int j = 0; j < P; ++j) {
       const int b = static_cast<int>((static_cast<u64>(ua[j]) * M) >> 32);
       const u64 c = (static_cast<u64>(ub[j]) * Q2) >> 32;
-      anc[j] = c < S.prob[b] ? b : S.alias[b];
+      if constexpr (C::PROB32) {
+        const uint32_t* p32 = reinterpret_cast<const uint32_t*>(S.prob);
+        anc[j] = static_cast<uint32_t>(c) < p32[b] ? b : reinterpret_cast<const uint16_t*>(p32 + M)[b];
+      } else {
+        anc[j] = c < S.prob[b] ? b : S.alias[b];
+      }
     }
   }
 }
@@ -889,7 +902,7 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
   S.scan = reinterpret_cast<u64*>(gs + C::g_scan);
   S.prob = reinterpret_cast<u64*>(gs + C::g_prob);
   S.alias = reinterpret_cast<int*>(gs + C::g_alias);
-  S.lists = reinterpret_cast<int*>(gs + C::g_lists);
+  S.lists = nullptr;   // per sub-filter: the stage's log-weight row
   uint2* bzw_s = reinterpret_cast<uint2*>(gs + C::g_scan);       // STAGED: Philox words after the resample
   volatile unsigned int* next_s = reinterpret_cast<unsigned int*>(gs + C::g_bar + 16);
   GroupCtx G;
@@ -980,6 +993,7 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
     }
     float* xs = reinterpret_cast<float*>(gs + C::g_stage + st * C::stage_bytes);
     float* ws = xs + D * M;
+    S.lists = reinterpret_cast<int*>(ws);   // Vose lists: the log-weight row is read into registers by then
     const long long gsf = P.g0 + n;                    // global sub-filter
     const uint32_t pbase = static_cast<uint32_t>(gsf * M);
     float* gblk = P.parts + n * C::ROW;                // this sub-filter's block in HBM
@@ -1605,7 +1619,7 @@ __global__ void __launch_bounds__(C::T* C::S) pf_resample_debug_kernel(const uin
   S.scan = reinterpret_cast<u64*>(gs + C::g_scan);
   S.prob = reinterpret_cast<u64*>(gs + C::g_prob);
   S.alias = reinterpret_cast<int*>(gs + C::g_alias);
-  S.lists = reinterpret_cast<int*>(gs + C::g_lists);
+  S.lists = reinterpret_cast<int*>(gs + C::g_stage);   // (no particle stage in the test hook)
   GroupCtx G;
   G.g = g;
   G.t = threadIdx.x - g * C::T;
