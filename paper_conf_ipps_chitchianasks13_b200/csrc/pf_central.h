@@ -35,10 +35,10 @@ struct CentralParams {
   int publish;   // only the argmax / record of the set in `in` (checkpoint restore)
   // Vose (resampler 1): the alias table over all M slots (sweep closed form, R10)
   int vose;
-  unsigned long long* dl;          // [M] per-tile inclusive deficit sums over the small slots
-  uint32_t* cn;                    // [M] per-tile inclusive small-slot counts
+  unsigned long long* vscal;       // [3] nL, D_last, Q (vz_lists -> vz_merge)
+  uint32_t* q32;                   // [M] integer weights q (u32)
   int* lists;                      // [M] small slots ascending, then large slots ascending
-  unsigned long long* vals;        // [M] D over the small list, then E over the large list
+  unsigned long long* vals;        // [M] exclusive D over the small list, then inclusive E over the large list
   unsigned long long* prob;        // [M] alias-table threshold (units of Q / M)
   int* alias;                      // [M]
   unsigned long long* tile_cnt;    // [tiles] small count per tile, then its inclusive prefix

@@ -361,7 +361,7 @@ pf::CentralParams central_params(pf_handle* h, long long k) {
     const long long M = h->g.M_local, T = h->g.tiles;
     u64* v = aux + M + 2 * T;
     c.vose = 1;
-    c.dl = v;
+    c.vscal = v;
     c.vals = v + M;
     c.prob = v + 2 * M;
     c.tile_cnt = v + 3 * M;
@@ -369,7 +369,7 @@ pf::CentralParams central_params(pf_handle* h, long long k) {
     c.tile_D = v + 3 * M + 2 * T;
     c.tile_D_incl = v + 3 * M + 3 * T;
     uint32_t* w = reinterpret_cast<uint32_t*>(v + 3 * M + 4 * T);
-    c.cn = w;
+    c.q32 = w;
     c.lists = reinterpret_cast<int*>(w + M);
     c.alias = reinterpret_cast<int*>(w + 2 * M);
   }
