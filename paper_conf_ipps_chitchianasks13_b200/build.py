@@ -16,7 +16,7 @@ ROOT = os.path.dirname(HERE)
 LIB = os.path.join(HERE, "libpf_b200.so")
 BUILD = os.path.join(HERE, "build")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
-SOURCES = ["pf_runtime.cu", "pf_debug.cu", "pf_central.cu", "pf_mean.cu", "pf_inst_nj2.cu", "pf_inst_nj5.cu", "pf_inst_nj28.cu", "pf_inst_lg1.cu"]
+SOURCES = ["pf_runtime.cu", "pf_debug.cu", "pf_central.cu", "pf_mean.cu", "pf_inst_nj2.cu", "pf_inst_nj5.cu", "pf_inst_nj28.cu", "pf_inst_lg1.cu", "pf_inst_armg.cu"]
 HEADERS = ["pf_device.cuh", "pf_model.cuh", "pf_kernels.cuh", "pf_registry.h", "pf_central.h", "pf_mean.h"]
 FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17", "-fmad=false",
          "-Xcompiler", "-fPIC", "-Xptxas", "-v", "-I", os.path.join(ROOT, "include")]

@@ -100,6 +100,7 @@ struct StepParams {
   unsigned char* peer_blk[kMaxRanks];
   int rank, world;
   long long mb_parity;     // floats per mailbox parity (n_ext * tt * E), same on every rank
+  int d, nj;               // state dimension and joints (read by runtime-dimension models only)
   unsigned long long rv;   // peer rendezvous number of this launch (>= 1, +1 per peer-mode launch on every rank)
   unsigned long long peer_timeout_ns;   // give up waiting at the rendezvous after this long (status word)
   float zin[32];           // step inputs carried by the launch itself (host-input mode)
@@ -184,7 +185,7 @@ struct KCfg {
   static constexpr int ROW = (D + 1) * M;    // floats per sub-filter block
   static constexpr bool SCAN32 = (M <= 512);  // Q <= M 2^22 fits 32 bits
   static constexpr bool STAGED = UNR < P;    // rolled sample loop: per-slot values via smem
-  static constexpr bool X2 = X2_ && (P % 2 == 0);   // sample two particles at once (packed f32x2)
+  static constexpr bool X2 = X2_ && (P % 2 == 0) && !Model::RUNTIME;   // two particles at once (packed f32x2)
   static constexpr bool CHUNKED = Model::CHUNKED;   // runtime loop over joint chunks (pf_model.cuh)
   static_assert(P >= 1 && P * T == M, "M must be a multiple of the group size");
   static_assert(P <= 32, "exclusion masks are 32-bit");
@@ -727,14 +728,35 @@ struct SampleChunked2 {
   }
 };
 
+// Streamed sample + weight with RUNTIME dimensions (the generic arm): the
+// same Box–Muller pairing, Philox words and per-component arithmetic as
+// SampleStream, as a loop over pairs (block 0 words 2-3 supplied).
+template <class Model>
+struct SampleRuntime {
+  template <typename X, typename O>
+  __device__ __forceinline__ static void run(const ModelConsts& mc, int nj, const float* hsu, const float* z,
+                                             const X& x, NoiseGen& gen, typename Model::Acc& A, const O& out) {
+    const int d = nj + 4;
+    u32x4 blk = gen.blk;
+#pragma unroll 1
+    for (int q = 0; q < (d + 1) / 2; ++q) {
+      const int w = 2 + 2 * q;
+      if ((w & 3) == 0) blk = philox4x32_10_rk(gen.p, gen.k, 0u, static_cast<uint32_t>(w >> 2), gen.rk);
+      float z0, z1;
+      normal_pair((w & 3) == 2 ? blk.z : blk.x, (w & 3) == 2 ? blk.w : blk.y, z0, z1);
+      out(2 * q, Model::take_rt(2 * q, nj, mc, hsu, z, x, z0, A));
+      if (2 * q + 1 < d) out(2 * q + 1, Model::take_rt(2 * q + 1, nj, mc, hsu, z, x, z1, A));
+    }
+  }
+};
+
 // Peer transport, halo rows (reading R3/R4 and the halo plan of
 // distributed.py): ring — local sub-filter 0 -> the previous rank's row
 // n_local + 1, the last -> the next rank's row n_local; torus — the first grid
 // row -> the rank above, rows n_local + C + c, the last grid row -> the rank
 // below, rows n_local + c.  The rows' first t entries [logw, index bits, x],
 // copied by the last CTA (every row is complete; no code in the step loop).
-template <int E>
-__device__ void peer_halo_rows(const StepParams& P) {   // whole CTA (the last one)
+static __device__ void peer_halo_rows(const StepParams& P, int E) {   // whole CTA (the last one)
   const long long nl = P.n_local, par = static_cast<long long>(P.k & 1u) * P.mb_parity;
   const int per = P.t * E;                                  // the row's first t entries
   const long long Cc = P.topo == TOPO_RING ? 1 : P.C;       // rows per side
@@ -800,8 +822,7 @@ __device__ __forceinline__ void top_t_merge(u64& rk, u64& rl, u64 nk, u64 nl, in
 // All-to-All pool from the per-group best t (pool_cta rows of the groups
 // that processed a sub-filter: static first index gid0 < n_local): the best t
 // of those candidates, entries copied from the mailbox.  Whole CTA.
-template <int E>
-__device__ void pool_top_t_cta(const StepParams& P, float* out, u64* red, long long groups) {   // red: 66 u64
+static __device__ void pool_top_t_cta(const StepParams& P, float* out, u64* red, long long groups, int E) {   // red: 66 u64
   u64* red_k = red;
   u64* red_l = red + 33;
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5, nw = (blockDim.x + 31) >> 5;
@@ -846,8 +867,7 @@ __device__ void pool_top_t_cta(const StepParams& P, float* out, u64* red, long l
 // All-to-All pool (§VI-E): the best t of `count` mailbox entries
 // (entry e = row e / t, item e % t, E floats [logw, index bits, x]) by the
 // order key of R6, copied to out[0..t) in order.  Whole CTA; t rounds.
-template <int E>
-__device__ void pool_top_t(const StepParams& P, const float* mb, long long count, float* out, u64* pool_red) {
+static __device__ void pool_top_t(const StepParams& P, const float* mb, long long count, float* out, u64* pool_red, int E) {
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5, nw = (blockDim.x + 31) >> 5;
   u64 prev = ~0ull;
   for (int jb = 0; jb < P.t; ++jb) {
@@ -888,7 +908,17 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
   if (threadIdx.x == 0) atomicMin(&pf_tl2[0], tl_now());
 #endif
   using Model = typename C::Model;
-  constexpr int ZD = Model::ZD, UD = Model::UD, M = C::M, D = C::D, E = C::E, GW = C::GW, PP = C::P;
+  constexpr int M = C::M, GW = C::GW, PP = C::P;
+  // dimensions: compile-time for the compiled models; the generic arm
+  // (Model::RUNTIME) takes them from the launch (its shared-memory stage is
+  // sized for its largest state, the HBM block and mailbox entry are exact)
+  constexpr bool RT = Model::RUNTIME;
+  const int D = RT ? P.d : C::D;
+  const int E = D + 2;
+  const int ZD = RT ? P.nj + 2 : Model::ZD;
+  const int UD = RT ? P.nj : Model::UD;
+  const long long ROW = static_cast<long long>(D + 1) * M;                  // floats per HBM block
+  const uint32_t stage_bytes = RT ? static_cast<uint32_t>(sizeof(float) * ROW) : static_cast<uint32_t>(C::stage_bytes);
   extern __shared__ __align__(128) unsigned char smem[];
   float* z_s = reinterpret_cast<float*>(smem + C::c_zin);
   float* hsu_s = z_s + ZD;
@@ -932,9 +962,8 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
   auto issue = [&](int b, long long nn) {   // thread 0 only
     next_s[b] = static_cast<unsigned int>(nn < P.n_local ? nn : P.n_local);
     if (nn < P.n_local) {
-      mbar_arrive_expect_tx(bars + b, static_cast<uint32_t>(C::stage_bytes));
-      bulk_g2s(gs + C::g_stage + b * C::stage_bytes, P.parts + nn * C::ROW, static_cast<uint32_t>(C::stage_bytes),
-               bars + b);
+      mbar_arrive_expect_tx(bars + b, stage_bytes);
+      bulk_g2s(gs + C::g_stage + b * C::stage_bytes, P.parts + nn * ROW, stage_bytes, bars + b);
     } else {
       mbar_arrive(bars + b);
     }
@@ -988,7 +1017,7 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
       // sample loop; pull it from HBM into L2 now, so that load hits L2
       if (G.t == 0) {
         const long long nn = gstride + pending;
-        if (nn < P.n_local) bulk_prefetch_l2(P.parts + nn * C::ROW, static_cast<uint32_t>(C::stage_bytes));
+        if (nn < P.n_local) bulk_prefetch_l2(P.parts + nn * ROW, stage_bytes);
       }
     }
     float* xs = reinterpret_cast<float*>(gs + C::g_stage + st * C::stage_bytes);
@@ -996,7 +1025,7 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
     S.lists = reinterpret_cast<int*>(ws);   // Vose lists: the log-weight row is read into registers by then
     const long long gsf = P.g0 + n;                    // global sub-filter
     const uint32_t pbase = static_cast<uint32_t>(gsf * M);
-    float* gblk = P.parts + n * C::ROW;                // this sub-filter's block in HBM
+    float* gblk = P.parts + n * ROW;                   // this sub-filter's block in HBM
     bool issued = false;   // NSTAGE 1: next load already started (after the sample loop)
     auto release_stage = [&]() {   // all generic smem accesses to the stage done: start the next load
       fence_proxy_async_smem();
@@ -1236,7 +1265,8 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
     }
 
     TL(tl_res);
-    if (C::X2 && do_sample) {
+    if constexpr (C::X2) {
+     if (do_sample) {
       // ---- a9 gather (smem) + a1 RNG + a2 sample + a3 weight + a10 store,
       //      two particles (slots j, j+1 of this thread) at a time with the
       //      floating-point work packed (f32x2, bit-identical lane by lane)
@@ -1297,6 +1327,7 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
         reinterpret_cast<float*>(bzw_s)[2 * sa] = lo2(l);   // own slots, after their Philox words were read
         reinterpret_cast<float*>(bzw_s)[2 * sb] = hi2(l);
       }
+     }
     } else if (do_sample) {
       // ---- a9 gather (smem) + a1 RNG + a2 sample + a3 weight + a10 store,
       //      one particle at a time (coalesced rows: consecutive threads,
@@ -1329,7 +1360,11 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
         NoiseGen gen{pbase + static_cast<uint32_t>(s), P.k, P.rk, u32x4{0u, 0u, z2, z3}};
         typename Model::Acc A;
         // (one particle per thread: the unrolled chain measured as fast as the chunked one)
-        SampleStream<Model, 0>::run(P.mc, hsu_s, z_s, x, gen, A, [out](int c, float v) { out[c * M] = v; });
+        if constexpr (RT) {
+          SampleRuntime<Model>::run(P.mc, P.nj, hsu_s, z_s, x, gen, A, [out](int c, float v) { out[c * M] = v; });
+        } else {
+          SampleStream<Model, 0>::run(P.mc, hsu_s, z_s, x, gen, A, [out](int c, float v) { out[c * M] = v; });
+        }
         float l = Model::finish(P.mc, z_s, A);
         if (!resampled) l = cr + l;   // F12
         out[D * M] = l;
@@ -1453,7 +1488,7 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
         const u64 key = __ldcg(P.key_cur);
         const uint32_t gidx = 0xFFFFFFFFu - static_cast<uint32_t>(key);
         const long long col = static_cast<long long>(gidx) - P.g0 * M;
-        const float* blk = P.parts + (col / M) * C::ROW + (col % M);
+        const float* blk = P.parts + (col / M) * ROW + (col % M);
         if (tid < D) pool[2 + tid] = __ldcg(blk + tid * M);
         if (tid == 0) {
           pool[0] = unord_f32(static_cast<uint32_t>(key >> 32));
@@ -1462,15 +1497,15 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
       } else {
         // reduction scratch: group 0's stage buffer (no load in flight after the loop)
         u64* red = reinterpret_cast<u64*>(smem + C::c_groups + C::g_stage);
-        if (P.pool_cta) pool_top_t_cta<E>(P, pool, red, static_cast<long long>(gridDim.x) * C::S);
-        else pool_top_t<E>(P, P.mb_cur, P.n_local * P.t, pool, red);
+        if (P.pool_cta) pool_top_t_cta(P, pool, red, static_cast<long long>(gridDim.x) * C::S, E);
+        else pool_top_t(P, P.mb_cur, P.n_local * P.t, pool, red, E);
       }
     }
     if (mode != MODE_EXCHANGE) {
       const u64 key = __ldcg(P.key_cur);
       const uint32_t gidx = 0xFFFFFFFFu - static_cast<uint32_t>(key);
       const long long col = static_cast<long long>(gidx) - P.g0 * M;
-      const float* blk = P.parts + (col / M) * C::ROW + (col % M);
+      const float* blk = P.parts + (col / M) * ROW + (col % M);
       float* outs[3] = {P.record, P.est_out, P.record_host};
       if (P.peer_mb[0] && (mode == MODE_STEP || mode == MODE_PUBLISH)) {
         // peer transport: the boundary sub-filters' best-t rows into the
@@ -1488,7 +1523,7 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
             peer_pool(P.peer_blk[r], par, P.rank)[e] = __ldcg(lp + e);
           }
         } else {
-          peer_halo_rows<E>(P);
+          peer_halo_rows(P, E);
         }
         if (tid < D) {
           const float v = __ldcg(blk + tid * M);

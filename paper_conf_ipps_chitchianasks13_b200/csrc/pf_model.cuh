@@ -63,6 +63,7 @@ struct ArmPlanar {
   static constexpr int kId = MODEL_ARM_PLANAR;
   static constexpr int NJ = NJ_;
   static constexpr int D = NJ + 4, ZD = NJ + 2, UD = NJ;
+  static constexpr bool RUNTIME = false;   // dimensions fixed at compile time
   // large states (the high-DOF arm): the joint chain runs as a loop over
   // chunks of four joints instead of being unrolled d times, so the
   // per-particle code fits the instruction cache (ncu: no_instruction stalls)
@@ -172,6 +173,51 @@ struct ArmPlanar {
   }
 };
 
+// --------------------------------------------- the generic (runtime) arm ---
+// The arm for ANY n_joints <= NJMAX (the fallback behind the compiled
+// instances n_j in {2, 5, 28}): the same F8–F10 arithmetic in the same order
+// as ArmPlanar<n_j>, with the joint count a runtime value (take_rt, one
+// component at a time; SampleRuntime in pf_kernels.cuh pairs the normals),
+// so its results are bit-identical to a compiled instance of that n_j.  The
+// kernel's shared-memory stage is sized for NJMAX + 4 components; the HBM
+// block and mailbox entries use the runtime d.  One particle per thread.
+template <int NJMAX_>
+struct ArmDyn {
+  static constexpr int kId = MODEL_ARM_PLANAR;
+  static constexpr int NJ = NJMAX_;                      // (the largest supported)
+  static constexpr int D = NJMAX_ + 4, ZD = NJMAX_ + 2, UD = NJMAX_;   // upper bounds
+  static constexpr bool RUNTIME = true;
+  static constexpr bool CHUNKED = false;
+  static constexpr int NC = 0;
+  using Acc = ArmAcc;
+  using Acc2 = ArmAcc2;
+  template <typename X>
+  __device__ __forceinline__ static float take_rt(int c, int nj, const ModelConsts& mc, const float* hs_u, const float* z,
+                                                  const X& x, float xi, Acc& A) {
+    if (c < nj) {
+      const float th = __fmaf_rn(mc.s_th, xi, x(c) + hs_u[c]);
+      A.phi = A.phi + th;                               // F9
+      sincos_c(A.phi, A.s, A.c);
+      A.px = __fmaf_rn(mc.lj, A.c, A.px);
+      A.py = __fmaf_rn(mc.lj, A.s, A.py);
+      const float r = (z[2 + c] - th) * mc.inv_thm;     // F10, joint residuals first
+      A.acc = (c == 0) ? r * r : __fmaf_rn(r, r, A.acc);
+      return th;
+    } else if (c == nj) {
+      A.xn = __fmaf_rn(mc.s_pos, xi, __fmaf_rn(mc.hs, x(nj + 2), x(nj)));
+      return A.xn;
+    } else if (c == nj + 1) {
+      A.yn = __fmaf_rn(mc.s_pos, xi, __fmaf_rn(mc.hs, x(nj + 3), x(nj + 1)));
+      return A.yn;
+    } else {
+      return __fmaf_rn(mc.s_vel, xi, x(c));
+    }
+  }
+  __device__ __forceinline__ static float finish(const ModelConsts& mc, const float* z, const Acc& A) {
+    return ArmPlanar<1>::finish(mc, z, A);   // camera frame + residuals: independent of n_j
+  }
+};
+
 // ------------------------------------------------- 1-D linear Gaussian ---
 // The linear-Gaussian special case of SURVEY §8(c) whole-filter pin (ii): one
 // joint of the arm with its angle sensor and no camera —
@@ -190,6 +236,7 @@ struct LinearGauss1D {
   static constexpr int kId = MODEL_LINEAR_GAUSS_1D;
   static constexpr int NJ = 1;   // (one "joint")
   static constexpr int D = 1, ZD = 1, UD = 1;
+  static constexpr bool RUNTIME = false;
   static constexpr bool CHUNKED = false;
   static constexpr int NC = 0;
   using Acc = LgAcc;

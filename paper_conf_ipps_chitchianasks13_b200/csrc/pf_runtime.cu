@@ -43,13 +43,15 @@ Table tables(int i) {
     case 0: return {pf::kEntriesNJ2, pf::kNumEntriesNJ2};
     case 1: return {pf::kEntriesNJ5, pf::kNumEntriesNJ5};
     case 2: return {pf::kEntriesNJ28, pf::kNumEntriesNJ28};
-    default: return {pf::kEntriesLG1, pf::kNumEntriesLG1};
+    case 3: return {pf::kEntriesLG1, pf::kNumEntriesLG1};
+    default: return {pf::kEntriesARMG, pf::kNumEntriesARMG};   // last: compiled n_j come first
   }
 }
-constexpr int kTables = 4;
+constexpr int kTables = 5;
+constexpr int kMaxGenericNJ = 28;   // the generic arm's stage holds d <= 32
 
 bool matches(const pf::KernelEntry& e, int model, int nj, int m, int res) {
-  return e.model == model && (model != PF_MODEL_ARM_PLANAR || e.nj == nj) && e.m == m && e.res == res;
+  return e.model == model && (model != PF_MODEL_ARM_PLANAR || e.nj == nj || e.nj == 0) && e.m == m && e.res == res;
 }
 
 // First entry matching (model, nj, m, res), or the PF_VARIANT-th one if set.
@@ -107,6 +109,7 @@ pf_status validate(const pf_config* cfg, const pf_model_params* mp, Geometry* g)
   if (!cfg || !mp) return PF_EINVAL;
   if (mp->model == PF_MODEL_ARM_PLANAR) {
     if (mp->n_joints < 1) return PF_EINVAL;
+    if (mp->n_joints > kMaxGenericNJ) return PF_EUNSUPPORTED;
     if (!(mp->sigma_cam > 0.0f) || !(mp->sigma_theta_meas > 0.0f) || !(mp->sigma_theta >= 0.0f) ||
         !(mp->sigma_pos >= 0.0f) || !(mp->sigma_vel >= 0.0f))
       return PF_EINVAL;
@@ -304,6 +307,8 @@ pf::StepParams base_params(pf_handle* h, long long k, int mode) {
   p.rank = h->cfg.rank;
   p.world = h->cfg.world;
   p.mb_parity = h->g.n_ext * h->g.tt * h->g.E;
+  p.d = h->g.d;
+  p.nj = h->g.nj;
   p.pool_cta = pool_cta_bytes(&h->cfg, h->g)
                    ? reinterpret_cast<u64*>(h->mailbox + 2 * h->g.n_ext * h->g.tt * h->g.E)
                    : nullptr;
@@ -1174,7 +1179,7 @@ int32_t pf_supported(int32_t* n_joints, int32_t* m, int32_t cap) {
   for (int ti = 0; ti < kTables; ++ti) {
     const Table t = tables(ti);
     for (int i = 0; i < t.n; ++i) {
-      if (t.e[i].model != PF_MODEL_ARM_PLANAR) continue;
+      if (t.e[i].model != PF_MODEL_ARM_PLANAR || t.e[i].nj == 0) continue;
       bool dup = false;
       for (int j = 0; j < i; ++j) dup = dup || (t.e[j].m == t.e[i].m && t.e[j].nj == t.e[i].nj);
       if (t.e[i].res != 0 || dup) continue;

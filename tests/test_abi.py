@@ -85,7 +85,13 @@ def test_invalid_configs(B, kw, code):
 
 def test_unsupported_model(B):
     out = B.pf_sizes()
-    assert B.lib().pf_query_sizes(C.byref(_cfg(B)), C.byref(_model(B, 7)), C.byref(out)) == B.PF_EUNSUPPORTED
+    # any n_joints <= 28 runs (compiled n_j in {2, 5, 28}, the generic arm for the rest); 29+ is not compiled
+    assert B.lib().pf_query_sizes(C.byref(_cfg(B)), C.byref(_model(B, 7)), C.byref(out)) == B.PF_OK
+    assert out.state == 4 * (7 + 4 + 1) * 16 * 64
+    assert B.lib().pf_query_sizes(C.byref(_cfg(B)), C.byref(_model(B, 29)), C.byref(out)) == B.PF_EUNSUPPORTED
+    # the centralized filter is compiled for n_j in {2, 5, 28} only
+    assert B.lib().pf_query_sizes(C.byref(_cfg(B, m=8192, n_filters=1, t=0, topo=0)), C.byref(_model(B, 7)),
+                                  C.byref(out)) == B.PF_EUNSUPPORTED
     assert (5, 256) in B.pf_supported() and (28, 256) in B.pf_supported()
     assert B.pf_strerror(B.PF_EINVAL).startswith("invalid")
 

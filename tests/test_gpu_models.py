@@ -118,3 +118,40 @@ def test_lg_streamed_batched_same(P, W):
     np.testing.assert_array_equal(a.get_particles()[0], b.get_particles()[0])
     a.close()
     b.close()
+
+
+@pytest.mark.parametrize("nj,m,N,topo,res", [(3, 64, 16, "ring", "rws"), (7, 128, 8, "torus", "vose"),
+                                             (12, 256, 4, "ring", "rws"), (1, 32, 8, "all2all", "rws"),
+                                             (20, 1024, 2, "ring", "vose")])
+def test_generic_arm_bit_exact(P, orc, W, nj, m, N, topo, res):
+    # any n_joints: the generic arm (runtime dimensions, pf_model.cuh ArmDyn)
+    # against the oracle, every step and the final set bit for bit
+    tr = W.make_trajectory(nj, 12, 2)
+    g = P.ParticleFilter(tr["mu0"], tr["sigma0"], P.ArmModel(n_joints=nj), m=m, n_filters=N, t=1, topo=topo,
+                         resampler=res, seed=11)
+    o = orc.Filter(orc.Config(m=m, n_filters=N, t=1, topo=topo, resampler=res, seed=11), orc.Model(n_joints=nj),
+                   tr["mu0"], tr["sigma0"])
+    for k in range(1, 13):
+        g.step(tr["Z"][k], tr["U"][k - 1])
+        o.step(tr["Z"][k], tr["U"][k - 1])
+        xg, lg, ig = g.estimate()
+        xo, lo, io = o.estimate()
+        assert ig == io, (k, ig, io)
+        np.testing.assert_array_equal(xg, xo)
+    sg, wg, _ = g.get_particles()
+    so, wo, _ = o.get()
+    np.testing.assert_array_equal(sg, so)
+    np.testing.assert_array_equal(wg, wo)
+    g.close()
+
+
+def test_generic_arm_sample_weight(P, orc, W):
+    nj = 9
+    tr = W.make_trajectory(nj, 6, 3)
+    g = P.ParticleFilter(tr["mu0"], tr["sigma0"], P.ArmModel(n_joints=nj), m=256, n_filters=8, seed=21)
+    s_in = W.random_particles(tr, 2048, 4)
+    sg, wg = g.debug_sample_weight(s_in, tr["Z"][2], tr["U"][1], 2)
+    so, wo = orc.sample_weight(orc.Model(n_joints=nj), 21, s_in, tr["Z"][2], tr["U"][1], 2)
+    np.testing.assert_array_equal(sg, so)
+    np.testing.assert_array_equal(wg, wo)
+    g.close()
