@@ -483,15 +483,13 @@ __global__ void __launch_bounds__(256) cz_draw_debug(const CentralParams C, cons
 template <class Model>
 __global__ void __launch_bounds__(256) cz_step(const CentralParams C) {
   constexpr int D = Model::D, ZD = Model::ZD, UD = Model::UD;
-  __shared__ f2 z2_s[ZD];
-  __shared__ f2 hsu2_s[UD];
+  __shared__ float z_s[ZD];
+  __shared__ float hsu_s[UD];
   __shared__ u64 red[32];
   __shared__ unsigned int s_last;
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  if (tid < ZD) z2_s[tid] = bc(C.z ? C.z[tid] : C.zin[tid]);
-  if (tid < UD) hsu2_s[tid] = bc(C.mc.hs * (C.u ? C.u[tid] : C.uin[tid]));   // control term h_s u_i (F8)
-  const ModelConsts2 mc2{bc(C.mc.lj), bc(C.mc.hs), bc(C.mc.s_th), bc(C.mc.s_pos), bc(C.mc.s_vel), bc(C.mc.inv_cam),
-                         bc(C.mc.inv_thm)};
+  if (tid < ZD) z_s[tid] = C.z ? C.z[tid] : C.zin[tid];
+  if (tid < UD) hsu_s[tid] = C.mc.hs * (C.u ? C.u[tid] : C.uin[tid]);   // control term h_s u_i (F8)
   const long long M = C.M;
   const int tiles = static_cast<int>(M / kCentralTile);
   __shared__ u64 tidx_s[kTidxMax];   // RWS: the inclusive tile prefix
@@ -502,40 +500,33 @@ __global__ void __launch_bounds__(256) cz_step(const CentralParams C) {
   __syncthreads();
   const u64 Q = C.first ? 0ull : C.tile_incl[tiles - 1];
   u64 best = 0ull;
-  // two adjacent particles per thread (M is a multiple of 4096): the sample
-  // and weight of the pair in packed f32x2 (bit-identical lane by lane), the
-  // rows stored as float2
-  for (long long i = 2 * (blockIdx.x * static_cast<long long>(blockDim.x) + tid); i < M;
-       i += 2 * static_cast<long long>(gridDim.x) * blockDim.x) {
-    const uint32_t pa = static_cast<uint32_t>(i), pb = pa + 1u;
+  // one particle per thread (grid-stride): the gather from random ancestors
+  // is latency-bound, so occupancy (registers) matters more than the packed
+  // pairs' instruction savings (measured: pairs at 74 registers no faster)
+  for (long long i = blockIdx.x * static_cast<long long>(blockDim.x) + tid; i < M;
+       i += static_cast<long long>(gridDim.x) * blockDim.x) {
+    const uint32_t p = static_cast<uint32_t>(i);
     if (C.publish) {   // restore: the loaded set is the step's weighted set
-      const float2 w = *reinterpret_cast<const float2*>(C.in + static_cast<long long>(D) * M + i);
-      const u64 ka = order_key(w.x, pa), kb = order_key(w.y, pb);
-      best = ka > best ? ka : best;
-      best = kb > best ? kb : best;
+      const u64 key = order_key(C.in[static_cast<long long>(D) * M + i], p);
+      best = key > best ? key : best;
       continue;
     }
-    const u32x4 b0a = philox4x32_10_rk(pa, C.k, 0u, 0u, C.rk);
-    const u32x4 b0b = philox4x32_10_rk(pb, C.k, 0u, 0u, C.rk);
-    const long long aa = C.first ? i : central_ancestor(C, Q, tiles, b0a.x, b0a.y, tidx);
-    const long long ab = C.first ? i + 1 : central_ancestor(C, Q, tiles, b0b.x, b0b.y, tidx);
-    const float* xa = C.in + aa;
-    const float* xb = C.in + ab;
-    auto x = [xa, xb, M](int c) { return pk(__ldg(xa + c * M), __ldg(xb + c * M)); };
-    NoiseGen2 gen{pa, pb, C.k, C.rk, u32x4{0u, 0u, b0a.z, b0a.w}, u32x4{0u, 0u, b0b.z, b0b.w}};
-    typename Model::Acc2 A;
+    const u32x4 b0 = philox4x32_10_rk(p, C.k, 0u, 0u, C.rk);
+    const long long a = C.first ? i : central_ancestor(C, Q, tiles, b0.x, b0.y, tidx);
+    const float* xa = C.in + a;
+    auto x = [xa, M](int c) { return __ldg(xa + c * M); };
+    NoiseGen gen{p, C.k, C.rk, u32x4{0u, 0u, b0.z, b0.w}};
+    typename Model::Acc A;
     float* out = C.out + i;
-    auto store2 = [out, M](int c, f2 v) { *reinterpret_cast<f2*>(out + c * M) = v; };
     if constexpr (Model::CHUNKED) {
-      SampleChunked2<Model>::run(mc2, hsu2_s, z2_s, x, gen, A, store2);
+      SampleChunked<Model>::run(C.mc, hsu_s, z_s, x, gen, A, [out, M](int c, float v) { out[c * M] = v; });
     } else {
-      SampleStream2<Model, 0>::run(mc2, hsu2_s, z2_s, x, gen, A, store2);
+      SampleStream<Model, 0>::run(C.mc, hsu_s, z_s, x, gen, A, [out, M](int c, float v) { out[c * M] = v; });
     }
-    const f2 l = Model::finish2(mc2, z2_s, A);
-    *reinterpret_cast<f2*>(out + static_cast<long long>(D) * M) = l;
-    const u64 ka = order_key(lo2(l), pa), kb = order_key(hi2(l), pb);
-    best = ka > best ? ka : best;
-    best = kb > best ? kb : best;
+    const float l = Model::finish(C.mc, z_s, A);
+    out[static_cast<long long>(D) * M] = l;
+    const u64 key = order_key(l, p);
+    best = key > best ? key : best;
   }
   // a5: block argmax -> one atomicMax; the last CTA copies the winner
   const u64 w = warp_max_u64(best);
