@@ -334,7 +334,7 @@ def test_error_behaviour(P, W):
     assert B.lib().pf_estimate(g.h, x.ctypes.data, None, None) == B.PF_OK
     assert B.pf_last_error(g.h) == B.PF_OK
     with pytest.raises(B.PFError):
-        P.ParticleFilter(tr["mu0"], tr["sigma0"], P.ArmModel(n_joints=3), m=64, n_filters=4)   # not compiled
+        P.ParticleFilter(tr["mu0"], tr["sigma0"], P.ArmModel(n_joints=29), m=64, n_filters=4)   # d > 32: not compiled
 
 
 @pytest.mark.parametrize("central", [False, True])
