@@ -472,8 +472,13 @@ __device__ __forceinline__ void resample_group(const uint32_t (&q)[C::P], const 
       small = a < Qg;
       Dinc = pinc[j] & ((1ull << 48) - 1);
       ls = static_cast<int>(pinc[j] >> 48) - (small ? 1 : 0);   // smalls before the slot
-      const u64 slot1 = static_cast<u64>(C::slot(G.t, j)) + 1;
-      Einc = Dinc + static_cast<u64>(M) * qinc[j] - slot1 * Qg;
+      const uint32_t slot1 = static_cast<uint32_t>(C::slot(G.t, j)) + 1u;
+      if constexpr (C::SCAN32) {   // Q < 2^32: 32 x 32 -> 64-bit products (one IMAD.WIDE each)
+        Einc = Dinc + static_cast<u64>(static_cast<uint32_t>(qinc[j])) * static_cast<uint32_t>(M) -
+               static_cast<u64>(slot1) * static_cast<uint32_t>(Qg);
+      } else {
+        Einc = Dinc + static_cast<u64>(M) * qinc[j] - static_cast<u64>(slot1) * Qg;
+      }
     };
     // Lists: small slots ascending with their EXCLUSIVE deficit sums A_i =
     // D_{i-1} (A_0 = 0) at [0, nL), large slots ascending with their
@@ -557,11 +562,12 @@ __device__ __forceinline__ void resample_group(const uint32_t (&q)[C::P], const 
 #pragma unroll
     for (int j = 0; j < P; ++j) {
       const int b = static_cast<int>((static_cast<u64>(ua[j]) * M) >> 32);
-      const u64 c = (static_cast<u64>(ub[j]) * Q2) >> 32;
-      if constexpr (C::PROB32) {
+      if constexpr (C::PROB32) {   // Q < 2^32: c = the high word of one 32 x 32 product
+        const uint32_t c = __umulhi(ub[j], static_cast<uint32_t>(Q2));
         const uint32_t* p32 = reinterpret_cast<const uint32_t*>(S.prob);
-        anc[j] = static_cast<uint32_t>(c) < p32[b] ? b : reinterpret_cast<const uint16_t*>(p32 + M)[b];
+        anc[j] = c < p32[b] ? b : reinterpret_cast<const uint16_t*>(p32 + M)[b];
       } else {
+        const u64 c = (static_cast<u64>(ub[j]) * Q2) >> 32;
         anc[j] = c < S.prob[b] ? b : S.alias[b];
       }
     }
