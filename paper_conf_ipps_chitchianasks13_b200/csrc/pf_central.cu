@@ -408,7 +408,7 @@ __device__ __forceinline__ long long first_greater(const u64* __restrict__ a, lo
 // memory, tidx, when it fits: kTidxMax tiles), then inside the tile in two
 // levels — every 64th inclusive sum first (6 probes), then the 64-slot block
 // (6 probes within 512 B) — the same first j with C_j > c as one search.
-constexpr int kTidxMax = 2048;   // tiles whose prefix a CTA keeps in shared memory (16 KB)
+constexpr int kTidxMax = 1024;   // tiles whose prefix a CTA keeps in shared memory (8 KB)
 __device__ __forceinline__ long long central_ancestor(const CentralParams& C, u64 Q, int tiles, uint32_t ua,
                                                       uint32_t ub, const u64* tidx) {
   if (C.vose) {
@@ -483,11 +483,14 @@ __global__ void __launch_bounds__(256) cz_draw_debug(const CentralParams C, cons
 template <class Model>
 __global__ void __launch_bounds__(256) cz_step(const CentralParams C) {
   constexpr int D = Model::D, ZD = Model::ZD, UD = Model::UD;
+  constexpr int S = central_stride(D);
   __shared__ float z_s[ZD];
   __shared__ float hsu_s[UD];
   __shared__ u64 red[32];
   __shared__ unsigned int s_last;
+  __shared__ float stage_s[256 / 32][32 * S];   // each warp's 32 new records, written out coalesced
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  float* st = stage_s[warp];
   if (tid < ZD) z_s[tid] = C.z ? C.z[tid] : C.zin[tid];
   if (tid < UD) hsu_s[tid] = C.mc.hs * (C.u ? C.u[tid] : C.uin[tid]);   // control term h_s u_i (F8)
   const long long M = C.M;
@@ -507,24 +510,33 @@ __global__ void __launch_bounds__(256) cz_step(const CentralParams C) {
        i += static_cast<long long>(gridDim.x) * blockDim.x) {
     const uint32_t p = static_cast<uint32_t>(i);
     if (C.publish) {   // restore: the loaded set is the step's weighted set
-      const u64 key = order_key(C.in[static_cast<long long>(D) * M + i], p);
+      const u64 key = order_key(C.lw_in[i], p);
       best = key > best ? key : best;
       continue;
     }
     const u32x4 b0 = philox4x32_10_rk(p, C.k, 0u, 0u, C.rk);
     const long long a = C.first ? i : central_ancestor(C, Q, tiles, b0.x, b0.y, tidx);
-    const float* xa = C.in + a;
-    auto x = [xa, M](int c) { return __ldg(xa + c * M); };
+    // AoS records: the ancestor's d components are one contiguous run (two
+    // or three sectors), not d rows M apart
+    const float* xa = C.in + a * S;
+    auto x = [xa](int c) { return __ldg(xa + c); };
     NoiseGen gen{p, C.k, C.rk, u32x4{0u, 0u, b0.z, b0.w}};
     typename Model::Acc A;
-    float* out = C.out + i;
+    float* rec = st + lane * S;
     if constexpr (Model::CHUNKED) {
-      SampleChunked<Model>::run(C.mc, hsu_s, z_s, x, gen, A, [out, M](int c, float v) { out[c * M] = v; });
+      SampleChunked<Model>::run(C.mc, hsu_s, z_s, x, gen, A, [rec](int c, float v) { rec[c] = v; });
     } else {
-      SampleStream<Model, 0>::run(C.mc, hsu_s, z_s, x, gen, A, [out, M](int c, float v) { out[c * M] = v; });
+      SampleStream<Model, 0>::run(C.mc, hsu_s, z_s, x, gen, A, [rec](int c, float v) { rec[c] = v; });
     }
     const float l = Model::finish(C.mc, z_s, A);
-    out[static_cast<long long>(D) * M] = l;
+    C.lw_out[i] = l;
+    // the warp's 32 consecutive records (i - lane .. i - lane + 31; M is a
+    // multiple of the grid stride's 32-aligned warps) as contiguous stores
+    __syncwarp();
+    float* dst = C.out + (i - lane) * S;
+#pragma unroll
+    for (int f = lane; f < 32 * S; f += 32) dst[f] = st[f];
+    __syncwarp();
     const u64 key = order_key(l, p);
     best = key > best ? key : best;
   }
@@ -547,7 +559,7 @@ __global__ void __launch_bounds__(256) cz_step(const CentralParams C) {
     float* outs[3] = {C.record, C.est_out, C.record_host};
     const float* src = C.publish ? C.in : C.out;
     if (tid < D) {
-      const float v = __ldcg(src + static_cast<long long>(tid) * M + gidx);
+      const float v = __ldcg(src + static_cast<long long>(gidx) * S + tid);
       for (int o = 0; o < 3; ++o)
         if (outs[o]) outs[o][4 + tid] = v;
     }
@@ -581,7 +593,7 @@ template <class Model>
 cudaError_t central_step_m(const CentralParams& c, int grid, cudaStream_t s) {
   const int tiles = static_cast<int>(c.M / kCentralTile);
   if (!c.first && !c.publish) {
-    const float* logw = c.in + static_cast<long long>(Model::D) * c.M;
+    const float* logw = c.lw_in;
     if (c.vose) {
       vz_q<<<tiles, kVThreads, 0, s>>>(logw, c.record_prev, nullptr, c.q32, c.tile_sum);
       vose_table(c, s);

@@ -9,11 +9,16 @@
 namespace pf {
 
 constexpr int kCentralTile = 4096;   // particles per scan tile (M must be a multiple)
+// floats per particle record of the centralized filter's AoS state buffers:
+// d rounded up to even (8-byte aligned records)
+__host__ __device__ constexpr int central_stride(int d) { return (d + 1) & ~1; }
 
 struct CentralParams {
   ModelConsts mc;           // model constants (pf_model.cuh)
-  const float* in;          // [D+1][M] weighted set of step k-1 (buffer (k-1)&1)
-  float* out;               // [D+1][M] step k (buffer k&1)
+  const float* in;          // [M][S] states of step k-1 (AoS records, S = central_stride(D); buffer (k-1)&1)
+  float* out;               // [M][S] states of step k (buffer k&1)
+  const float* lw_in;       // [M] log-weights of step k-1
+  float* lw_out;            // [M] log-weights of step k
   long long M;
   unsigned long long* cl;   // [M] per-tile inclusive sums of q
   unsigned long long* tile_sum;    // [M / tile]

@@ -25,10 +25,13 @@ namespace {
 
 typedef unsigned long long u64;
 
+// D: the state dimension (compiled d) or an upper bound with the runtime d
+// in dr (the generic arm: components c >= dr contribute 0 and are not stored)
 template <int D>
 __global__ void __launch_bounds__(kMeanThreads) mean_partial_kernel(const float* __restrict__ parts, long long n_blocks,
                                                                     int m, long long row, const float* record,
-                                                                    double* __restrict__ partials) {
+                                                                    double* __restrict__ partials, int aos,
+                                                                    const float* __restrict__ lw, int dr) {
   __shared__ double sm[kMeanThreads / 32][D + 1];
   const float L = record[2];   // log-weight of the (global) best particle
   const long long total = n_blocks * m;
@@ -39,13 +42,15 @@ __global__ void __launch_bounds__(kMeanThreads) mean_partial_kernel(const float*
   for (long long p = blockIdx.x * static_cast<long long>(blockDim.x) + threadIdx.x; p < total;
        p += static_cast<long long>(gridDim.x) * blockDim.x) {
     const long long n = p / m, i = p - n * m;
-    const float* b = parts + n * row + i;
-    const uint32_t q = expq_c(__ldg(b + static_cast<long long>(D) * m) - L);
+    const float* b = aos ? parts + p * aos : parts + n * row + i;
+    const long long cs = aos ? 1 : m;   // component stride
+    const uint32_t q = expq_c((aos ? __ldg(lw + p) : __ldg(b + static_cast<long long>(dr) * m)) - L);
     if (q) {
       Q += q;
       const double qd = static_cast<double>(q);
 #pragma unroll
-      for (int c = 0; c < D; ++c) S[c] = fma(qd, static_cast<double>(__ldg(b + static_cast<long long>(c) * m)), S[c]);
+      for (int c = 0; c < D; ++c)
+        if (c < dr) S[c] = fma(qd, static_cast<double>(__ldg(b + c * cs)), S[c]);
     }
   }
 #pragma unroll
@@ -61,9 +66,9 @@ __global__ void __launch_bounds__(kMeanThreads) mean_partial_kernel(const float*
     for (int c = 0; c < D; ++c) sm[warp][1 + c] = S[c];
   }
   __syncthreads();
-  if (threadIdx.x <= D) {
+  if (threadIdx.x <= dr) {
     const int c = threadIdx.x;
-    double* out = partials + static_cast<long long>(blockIdx.x) * (D + 1);
+    double* out = partials + static_cast<long long>(blockIdx.x) * (dr + 1);
     if (c == 0) {
       u64 t = 0;
       for (int w = 0; w < kMeanThreads / 32; ++w) t += static_cast<u64>(__double_as_longlong(sm[w][0]));
@@ -102,17 +107,19 @@ __global__ void mean_final_kernel(const double* __restrict__ partials, int count
 }
 
 cudaError_t mean_partials(const MeanParams& mp, cudaStream_t s) {
+#define PF_MEAN(DD) mean_partial_kernel<DD><<<kMeanGrid, kMeanThreads, 0, s>>>(mp.parts, mp.n_blocks, mp.m, mp.row, \
+                                                                          mp.record, mp.partials, mp.aos_stride, mp.lw, mp.d)
   switch (mp.d) {
-    case 1: mean_partial_kernel<1><<<kMeanGrid, kMeanThreads, 0, s>>>(mp.parts, mp.n_blocks, mp.m, mp.row, mp.record,
-                                                                       mp.partials); break;   // linear-Gaussian model
-    case 6: mean_partial_kernel<6><<<kMeanGrid, kMeanThreads, 0, s>>>(mp.parts, mp.n_blocks, mp.m, mp.row, mp.record,
-                                                                       mp.partials); break;
-    case 9: mean_partial_kernel<9><<<kMeanGrid, kMeanThreads, 0, s>>>(mp.parts, mp.n_blocks, mp.m, mp.row, mp.record,
-                                                                       mp.partials); break;
-    case 32: mean_partial_kernel<32><<<kMeanGrid, kMeanThreads, 0, s>>>(mp.parts, mp.n_blocks, mp.m, mp.row,
-                                                                         mp.record, mp.partials); break;
-    default: return cudaErrorInvalidValue;
+    case 1: PF_MEAN(1); break;   // the linear-Gaussian model
+    case 6: PF_MEAN(6); break;
+    case 9: PF_MEAN(9); break;
+    case 32: PF_MEAN(32); break;
+    default:
+      if (mp.d < 1 || mp.d > 32) return cudaErrorInvalidValue;
+      if (mp.d <= 12) PF_MEAN(12);   // the generic arm (runtime d)
+      else PF_MEAN(32);
   }
+#undef PF_MEAN
   return cudaGetLastError();
 }
 

@@ -13,6 +13,8 @@ struct MeanParams {
   int m;                // particles per block
   int d;                // state dimension (1, 6, 9 or 32)
   long long row;        // floats per block, (d+1) m
+  int aos_stride;       // > 0: AoS records parts[p * aos_stride + c] and log-weights lw[p] (the centralized filter)
+  const float* lw;
   const float* record;  // estimate record: record[2] = log-weight of the (global) best particle
   double* partials;     // [kMeanGrid][d+1] scratch
 };

@@ -340,16 +340,28 @@ void host_inputs(pf_handle* h, pf::StepParams& p, const float* z, const float* u
   std::memcpy(p.uin, u, sizeof(float) * h->g.ud);
 }
 
-// Centralized filter: particle buffers ping-pong ([2][D+1][M]), then the
-// per-particle tile sums (u64 [M]) and two u64 arrays of tile totals.
-// Vose adds per slot dl, vals, prob (u64) and cn, lists, alias (32-bit), and
-// four u64 arrays of tile totals / prefixes.
+// Centralized filter: AoS state records ping-pong ([2][M][S], S =
+// central_stride(d): the random-ancestor gather reads one contiguous record),
+// then the log-weights ping-pong ([2][M]), then the per-particle tile sums
+// (u64 [M]) and two u64 arrays of tile totals.  Vose adds per slot vscal,
+// vals, prob (u64) and q32, lists, alias (32-bit), and four u64 arrays of
+// tile totals / prefixes.
+long long central_S(const Geometry& g) { return pf::central_stride(g.d); }
+long long central_floats(const Geometry& g) { return 2 * g.M_local * central_S(g) + 2 * g.M_local; }
 size_t central_bytes(const Geometry& g) {
   const size_t vose = g.vose ? sizeof(u64) * (3 * g.M_local + 4 * g.tiles) + sizeof(uint32_t) * 3 * g.M_local : 0;
-  return sizeof(float) * 2 * g.ROW + sizeof(u64) * (g.M_local + 2 * g.tiles) + vose;
+  return sizeof(float) * central_floats(g) + sizeof(u64) * (g.M_local + 2 * g.tiles) + vose;
 }
-// weighted set of step k lives in particle buffer (central: k & 1; else the only one)
-float* set_of_step(pf_handle* h, long long k) { return h->parts + (h->g.central ? (k & 1) * h->g.ROW : 0); }
+// weighted set of step k lives in particle buffer (central: the state records of buffer k & 1; else
+// the only blocked SoA buffer)
+float* set_of_step(pf_handle* h, long long k) {
+  return h->parts + (h->g.central ? (k & 1) * h->g.M_local * central_S(h->g) : 0);
+}
+// central: the log-weights that go with the state buffer `state`
+float* central_lw_of(pf_handle* h, const float* state) {
+  const long long idx = (state - h->parts) / (h->g.M_local * central_S(h->g));
+  return h->parts + 2 * h->g.M_local * central_S(h->g) + idx * h->g.M_local;
+}
 
 pf::CentralParams central_params(pf_handle* h, long long k) {
   pf::CentralParams c;
@@ -357,8 +369,10 @@ pf::CentralParams central_params(pf_handle* h, long long k) {
   c.mc = h->mc;
   c.in = set_of_step(h, k - 1);
   c.out = set_of_step(h, k);
+  c.lw_in = central_lw_of(h, c.in);
+  c.lw_out = central_lw_of(h, c.out);
   c.M = h->g.M_local;
-  u64* aux = reinterpret_cast<u64*>(h->parts + 2 * h->g.ROW);
+  u64* aux = reinterpret_cast<u64*>(h->parts + central_floats(h->g));
   c.cl = aux;
   c.tile_sum = aux + h->g.M_local;
   c.tile_incl = aux + h->g.M_local + h->g.tiles;
@@ -419,14 +433,17 @@ void host_inputs(pf_handle* h, pf::CentralParams& c, const float* z, const float
 }
 
 __global__ void pf_init_kernel(float* parts, int m, long long M_local, uint32_t p0, int d, const float* mu0,
-                               const float* s0, uint32_t key0, uint32_t key1) {
+                               const float* s0, uint32_t key0, uint32_t key1, int aos_stride, float* aos_lw) {
   // F11: x_c = fma(sigma0_c, xi_c, mu0_c); pair q of particle p from words
   // 2(q&1), 2(q&1)+1 of Philox (p, 0, 2, q>>1) (R13, stream 2 = init).
+  // Layout: blocked SoA [n][d+1][m]; the centralized filter (aos_stride > 0):
+  // AoS records [M][aos_stride] + log-weights aos_lw [M].
   const long long row = static_cast<long long>(d + 1) * m;
   for (long long col = blockIdx.x * static_cast<long long>(blockDim.x) + threadIdx.x; col < M_local;
        col += static_cast<long long>(gridDim.x) * blockDim.x) {
     const uint32_t p = p0 + static_cast<uint32_t>(col);
-    float* blk = parts + (col / m) * row + (col % m);
+    const long long cs = aos_stride ? 1 : m;   // component stride
+    float* blk = aos_stride ? parts + col * aos_stride : parts + (col / m) * row + (col % m);
     pf::u32x4 blk4{0, 0, 0, 0};
     for (int q = 0; q < (d + 1) / 2; ++q) {
       if ((q & 1) == 0) blk4 = pf::philox4x32_10(p, 0u, 2u, static_cast<uint32_t>(q >> 1), key0, key1);
@@ -435,10 +452,11 @@ __global__ void pf_init_kernel(float* parts, int m, long long M_local, uint32_t 
       float z0, z1;
       pf::normal_pair(x0, x1, z0, z1);
       const int c = 2 * q;
-      blk[c * m] = __fmaf_rn(s0[c], z0, mu0[c]);
-      if (c + 1 < d) blk[(c + 1) * m] = __fmaf_rn(s0[c + 1], z1, mu0[c + 1]);
+      blk[c * cs] = __fmaf_rn(s0[c], z0, mu0[c]);
+      if (c + 1 < d) blk[(c + 1) * cs] = __fmaf_rn(s0[c + 1], z1, mu0[c + 1]);
     }
-    blk[d * m] = 0.0f;
+    if (aos_stride) aos_lw[col] = 0.0f;
+    else blk[d * m] = 0.0f;
   }
 }
 
@@ -625,7 +643,8 @@ pf_status pf_init(const pf_config* cfg, const pf_model_params* model, const pf_b
     pf_init_kernel<<<static_cast<int>(blocks < 8 * sms ? blocks : 8 * sms), 256, 0, h->stream>>>(
         h->parts, g.m, g.M_local, static_cast<uint32_t>(g.g0 * g.m), g.d,
         reinterpret_cast<const float*>(h->scratch + kOffMu0), reinterpret_cast<const float*>(h->scratch + kOffSigma0),
-        static_cast<uint32_t>(cfg->seed), static_cast<uint32_t>(cfg->seed >> 32));
+        static_cast<uint32_t>(cfg->seed), static_cast<uint32_t>(cfg->seed >> 32),
+        g.central ? static_cast<int>(central_S(g)) : 0, g.central ? central_lw_of(h, h->parts) : nullptr);
     e = cudaGetLastError();
   }
   // the prior copy reads a stack buffer: finish before returning
@@ -768,6 +787,8 @@ static pf_status mean_partials_launch(pf_handle* h) {
   mp.m = h->g.central ? static_cast<int>(h->g.M_local) : h->g.m;
   mp.d = h->g.d;
   mp.row = h->g.ROW;
+  mp.aos_stride = h->g.central ? static_cast<int>(central_S(h->g)) : 0;
+  mp.lw = h->g.central ? central_lw_of(h, mp.parts) : nullptr;
   mp.record = record(h);
   mp.partials = mean_scratch(h);
   return sticky(h, pf::mean_partials(mp, h->stream));
@@ -870,6 +891,7 @@ static pf_status publish(pf_handle* h, long long step) {
   if (h->g.central) {
     pf::CentralParams c = central_params(h, step);
     c.in = set_of_step(h, step);
+    c.lw_in = central_lw_of(h, c.in);
     c.publish = 1;
     return launch_central(h, c);
   }
@@ -1197,6 +1219,20 @@ int32_t pf_supported(int32_t* n_joints, int32_t* m, int32_t cap) {
 
 namespace {
 cudaError_t rows_to_device(pf_handle* h, float* base, const float* host, int row0, int nrows) {
+  if (h->g.central) {   // AoS records + the log-weight array (transposed on the host)
+    const long long M = h->g.M_local, S = central_S(h->g);
+    const int d = h->g.d;
+    if (row0 == d && nrows == 1)
+      return cudaMemcpy(central_lw_of(h, base), host, sizeof(float) * M, cudaMemcpyHostToDevice);
+    if (row0 != 0 || nrows != d) return cudaErrorInvalidValue;
+    float* tmp = static_cast<float*>(std::calloc(static_cast<size_t>(M * S), sizeof(float)));
+    if (!tmp) return cudaErrorMemoryAllocation;
+    for (int c = 0; c < d; ++c)
+      for (long long p = 0; p < M; ++p) tmp[p * S + c] = host[c * M + p];
+    const cudaError_t e = cudaMemcpy(base, tmp, sizeof(float) * M * S, cudaMemcpyHostToDevice);
+    std::free(tmp);
+    return e;
+  }
   const size_t m = h->g.m;
   for (int r = 0; r < nrows; ++r) {
     cudaError_t e = cudaMemcpy2D(base + (row0 + r) * m, sizeof(float) * h->g.ROW,
@@ -1207,6 +1243,21 @@ cudaError_t rows_to_device(pf_handle* h, float* base, const float* host, int row
   return cudaSuccess;
 }
 cudaError_t rows_to_host(pf_handle* h, const float* base, float* host, int row0, int nrows) {
+  if (h->g.central) {
+    const long long M = h->g.M_local, S = central_S(h->g);
+    const int d = h->g.d;
+    if (row0 == d && nrows == 1)
+      return cudaMemcpy(host, central_lw_of(h, base), sizeof(float) * M, cudaMemcpyDeviceToHost);
+    if (row0 != 0 || nrows != d) return cudaErrorInvalidValue;
+    float* tmp = static_cast<float*>(std::malloc(sizeof(float) * M * S));
+    if (!tmp) return cudaErrorMemoryAllocation;
+    const cudaError_t e = cudaMemcpy(tmp, base, sizeof(float) * M * S, cudaMemcpyDeviceToHost);
+    if (e == cudaSuccess)
+      for (int c = 0; c < d; ++c)
+        for (long long p = 0; p < M; ++p) host[c * M + p] = tmp[p * S + c];
+    std::free(tmp);
+    return e;
+  }
   const size_t m = h->g.m;
   for (int r = 0; r < nrows; ++r) {
     cudaError_t e = cudaMemcpy2D(host + static_cast<size_t>(r) * h->g.M_local, sizeof(float) * m,

@@ -145,10 +145,22 @@ class ParticleFilter:
     @property
     def particles(self) -> torch.Tensor:
         """Device particle blocks [n_local][d+1][m] (rows 0..d-1 state, row d log-weight).
-        Centralized filter: the buffer holding the current step's set (ping-pong, k & 1)."""
+        Centralized filter: the AoS state records [m][S] (S = d rounded up to even) of the
+        current step's buffer (ping-pong, k & 1); its log-weights are `central_logw`."""
+        if self.central:
+            S = (self.d + 1) & ~1
+            n = self.m * S
+            off = 4 * n * (self._k & 1)
+            return self._parts[off: off + 4 * n].view(torch.float32).view(self.m, S)
         n = self.shard.n_local * (self.d + 1) * self.m
-        off = 4 * n * (self._k & 1) if self.central else 0
-        return self._parts[off: off + 4 * n].view(torch.float32).view(self.shard.n_local, self.d + 1, self.m)
+        return self._parts[: 4 * n].view(torch.float32).view(self.shard.n_local, self.d + 1, self.m)
+
+    @property
+    def central_logw(self) -> torch.Tensor:
+        """Centralized filter: the log-weights [m] of the current step (device)."""
+        S = (self.d + 1) & ~1
+        off = 4 * (2 * self.m * S + (self._k & 1) * self.m)
+        return self._parts[off: off + 4 * self.m].view(torch.float32)
 
     @property
     def mailbox(self) -> torch.Tensor:

@@ -84,7 +84,8 @@ def test_central_resume_and_batch(P, orc, W):
         xo, lo, io = o.estimate()
         np.testing.assert_array_equal(est[k - 7, 4:].cpu().numpy(), xo)
     np.testing.assert_array_equal(g.get_particles()[0], o.get()[0])
-    np.testing.assert_array_equal(g.particles[0, :nj + 4].cpu().numpy(), o.get()[0])
+    np.testing.assert_array_equal(g.particles[:, :nj + 4].T.cpu().numpy(), o.get()[0])   # AoS records
+    np.testing.assert_array_equal(g.central_logw.cpu().numpy(), o.get()[1])
     g.close()
 
 
