@@ -27,7 +27,8 @@ def _close(a, b):
 
 
 @pytest.mark.parametrize("nj,m,N,topo,res", [(2, 64, 16, "ring", "rws"), (5, 256, 8, "torus", "vose"),
-                                             (28, 32, 8, "ring", "rws")])
+                                             (28, 32, 8, "ring", "rws"), (7, 64, 8, "ring", "rws"),
+                                             (15, 128, 4, "ring", "vose")])   # (+ the generic arm: d = 11, 19)
 def test_mean_estimate_trajectory(P, orc, W, nj, m, N, topo, res):
     T = 20
     tr = W.make_trajectory(nj, T, 0)
@@ -106,4 +107,18 @@ def test_mean_errors(P, W):
     g = P.ParticleFilter(tr["mu0"], tr["sigma0"], P.ArmModel(n_joints=5), m=64, n_filters=4)
     with pytest.raises(B.PFError):   # before the first step
         g.estimate_mean()
+    g.close()
+
+
+@pytest.mark.parametrize("res", ["rws", "vose"])
+def test_mean_central_aos(P, orc, W, res):
+    # the centralized filter's AoS records: the mean of the GPU's own set vs
+    # the oracle's weighted mean of that set (read back through get_particles)
+    tr = W.make_trajectory(5, 6, 2)
+    g = P.ParticleFilter(tr["mu0"], tr["sigma0"], P.ArmModel(n_joints=5), m=16384, n_filters=1, t=0, topo="none",
+                         resampler=res, seed=8)
+    for k in range(1, 5):
+        g.step(tr["Z"][k], tr["U"][k - 1])
+    s, w, _ = g.get_particles()
+    _close(g.estimate_mean(), orc.weighted_mean(s, w))
     g.close()
