@@ -56,4 +56,17 @@ for rep in range(3):
     bins = np.arange(0, span + 2000, 2000)
     busy = [int(np.sum((ready <= b + 1000) & (end > b + 1000))) for b in bins[:-1]]
     print("  busy sub-filters per 2 us:", busy)
+    if rep == 2:   # one machine-readable line (the Fig. 4-style per-phase breakdown)
+        import json
+        print("TIMELINE " + json.dumps({
+            "n_joints": nj, "m": m, "N": N, "particles": m * N, "resampler": res, "flush_l2": flush_l2,
+            "event_us": e0.elapsed_time(e1) * 1e3, "kernel_span_us": span / 1e3,
+            "epilogue_us": (int(t2[2]) - int(t2[1])) / 1e3, "first_data_us": ready.min() / 1e3,
+            "groups": int(len(np.unique(grp))), "sub_filters": n,
+            "per_sub_filter_us": {"wait": float(np.mean(ready - w0)) / 1e3, "exchange": float(np.mean(merged - ready)) / 1e3,
+                                  "normalise_resample": float(np.mean(resd - merged)) / 1e3,
+                                  "sample_weight_store": float(np.mean(smp - resd)) / 1e3,
+                                  "reduce_finish": float(np.mean(end - smp)) / 1e3},
+            "group_end_us": {"p10": ends[len(ends) // 10] / 1e3, "p50": ends[len(ends) // 2] / 1e3,
+                             "p90": ends[9 * len(ends) // 10] / 1e3, "max": ends[-1] / 1e3}}), flush=True)
 g.close()
