@@ -23,7 +23,11 @@
  *    [n_local][d+1][m] — for every local sub-filter one contiguous block
  *    whose rows 0..d-1 are the state components (d = n_joints + 4:
  *    theta_0..theta_{n_j-1}, x, y, v_x, v_y — PAPER.md:22 §VII-A) of its m
- *    particles and whose row d is their log-weight (reading R7).
+ *    particles and whose row d is their log-weight (reading R7).  The
+ *    centralized filter (n_filters == 1, m > 1024) instead keeps AoS records:
+ *    float [2][m][S] states (S = d rounded up to even; ping-pong by step
+ *    parity), then float [2][m] log-weights, then its resampling tables — so
+ *    the global resampler's random-ancestor gather reads one contiguous record.
  *  - Host layout (get/set/debug hooks): state float32 [d][M_local] (row c =
  *    component c of every local particle, column n_local*m + i for
  *    sub-filter n_local, slot i), log-weights float32 [M_local].
@@ -128,7 +132,8 @@ typedef struct {
 
 /* Bytes of each caller-owned device buffer. */
 typedef struct {
-  uint64_t state;    /* float [n_local][d+1][m]: states + log-weights (blocked SoA) */
+  uint64_t state;    /* float [n_local][d+1][m]: states + log-weights (blocked SoA); */
+                     /* centralized filter: AoS records + tables, see above        */
   uint64_t mailbox;  /* float [2][n_ext][max(t,1)][d+2]: exchange mailbox, see below */
   uint64_t scratch;  /* keys, counters, estimate record, step inputs                */
 } pf_sizes;
