@@ -1477,14 +1477,15 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
   __syncthreads();
   if (threadIdx.x == 0) {
     // the CTA barrier orders every thread's writes (mailbox rows, key) before
-    // thread 0's cumulative gpu-scope fence and the completion count
-    __threadfence();
-    const unsigned int prev = atomicAdd(P.counter, 1u);
+    // thread 0's completion count, a gpu-scope acquire-release RMW (cumulative:
+    // it releases what the barrier ordered before it, and the last CTA's
+    // acquire orders its reads below after every other CTA's release)
+    unsigned int prev;
+    asm volatile("atom.acq_rel.gpu.global.add.u32 %0, [%1], 1;" : "=r"(prev) : "l"(P.counter) : "memory");
     s_last = (prev == gridDim.x - 1) ? 1u : 0u;
   }
   __syncthreads();
   if (s_last) {
-    __threadfence();
     const int tid = threadIdx.x;
     // All-to-All: this shard's best t -> pool row pool_local_row (first: the
     // peer transport also ships it to every rank before the rendezvous)
