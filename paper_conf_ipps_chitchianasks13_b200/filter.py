@@ -179,10 +179,14 @@ class ParticleFilter:
         """One time step (host numpy z/u, or device tensors with device_inputs)."""
         if self._device_inputs:
             st = self._step_fn(self.h, z.data_ptr(), u.data_ptr())
-        else:   # copied into the launch by pf_step (R-contract: host inputs travel with the kernel)
-            np.copyto(self._zin, z, casting="same_kind")
-            np.copyto(self._uin, u, casting="same_kind")
-            st = self._step_fn(self.h, self._zin_p, self._uin_p)
+        else:   # copied into the launch by pf_step (host inputs travel with the kernel)
+            if (type(z) is np.ndarray and type(u) is np.ndarray and z.dtype == np.float32 and u.dtype == np.float32
+                    and z.flags.c_contiguous and u.flags.c_contiguous and z.size == self.zd and u.size == self.ud):
+                st = self._step_fn(self.h, z.ctypes.data, u.ctypes.data)   # no staging copy
+            else:
+                np.copyto(self._zin, z, casting="same_kind")
+                np.copyto(self._uin, u, casting="same_kind")
+                st = self._step_fn(self.h, self._zin_p, self._uin_p)
         if st != B.PF_OK:
             B.check(st, "pf_step")
         self._k += 1
