@@ -28,10 +28,13 @@ python scripts/ncu_opcodes.py gpurun_out/r02_prof_c5v.ncu-rep 16777216 40 > gpur
 python scripts/ncu_lines.py gpurun_out/r02_prof_c2.ncu-rep 50 > gpurun_out/r02_source_lines_c2.txt
 rm -f gpurun_out/r02_prof_c2v.ncu-rep gpurun_out/r02_prof_c5.ncu-rep gpurun_out/r02_prof_c5v.ncu-rep gpurun_out/r02_prof_c4.ncu-rep gpurun_out/r02_prof_c4rws.ncu-rep
 timeout 900 python scripts/sweeps.py > gpurun_out/r02_sweeps.jsonl 2> gpurun_out/r02_sweeps.err
+timeout 300 python scripts/sweeps.py central > gpurun_out/r02_central_sweep.jsonl 2>> gpurun_out/r02_sweeps.err
 for tool in memcheck racecheck synccheck initcheck; do
   echo "== compute-sanitizer --tool $tool --kernel-name kns=pf_ python scripts/sanitize_run.py"
   timeout 900 compute-sanitizer --tool $tool --kernel-name kns=pf_ python scripts/sanitize_run.py 2>&1 | grep -v "^\s*$"
 done > gpurun_out/r02_compute_sanitizer.txt 2>&1
+bash scripts/gcall_r02_timeline.sh > /dev/null 2>&1
+timeout 600 python scripts/accuracy_kalman.py > gpurun_out/r02_accuracy_kalman.jsonl 2> gpurun_out/r02_accuracy_kalman.err
 timeout 400 python -m torch.distributed.run --nnodes=1 --nproc-per-node 2 --master-addr 127.0.0.1 --master-port 29555 \
   bench.py --gpus 2 --steps 5 --warmup 3 --no-extras --cpu-seconds 1 > gpurun_out/r02_bench_2rank.json 2> gpurun_out/r02_bench_2rank.err
 ls -la gpurun_out | grep r02
