@@ -69,7 +69,9 @@ typedef enum { PF_RESAMPLE_RWS = 0, PF_RESAMPLE_VOSE = 1 } pf_resampler;
  *                            h(x) of reading R14; d = n_joints + 4, z has
  *                            n_joints + 2 entries (x_C, y_C, joint angles),
  *                            u has n_joints; compiled for n_joints in
- *                            {2, 5, 28} (others: PF_EUNSUPPORTED).
+ *                            {2, 5, 28}, any other n_joints <= 28 through the
+ *                            generic runtime-dimension arm (bit-identical);
+ *                            > 28: PF_EUNSUPPORTED.
  *  PF_MODEL_LINEAR_GAUSS_1D  one joint with its angle sensor and no camera:
  *                            theta_k = theta_{k-1} + h_s u + w,
  *                            w ~ N(0, sigma_theta^2); z = theta + v,

@@ -482,13 +482,18 @@ __global__ void __launch_bounds__(256) cz_draw_debug(const CentralParams C, cons
 
 template <class Model>
 __global__ void __launch_bounds__(256) cz_step(const CentralParams C) {
-  constexpr int D = Model::D, ZD = Model::ZD, UD = Model::UD;
-  constexpr int S = central_stride(D);
-  __shared__ float z_s[ZD];
-  __shared__ float hsu_s[UD];
+  // dimensions: compile-time, or from the launch for the generic arm
+  // (Model::RUNTIME: the stage is sized for its largest d, records use the runtime d)
+  constexpr bool RT = Model::RUNTIME;
+  constexpr int SMAX = central_stride(Model::D);
+  const int D = RT ? C.d : Model::D;
+  const int S = RT ? central_stride(C.d) : SMAX;
+  const int ZD = RT ? C.nj + 2 : Model::ZD, UD = RT ? C.nj : Model::UD;
+  __shared__ float z_s[Model::ZD];
+  __shared__ float hsu_s[Model::UD];
   __shared__ u64 red[32];
   __shared__ unsigned int s_last;
-  __shared__ float stage_s[256 / 32][32 * S];   // each warp's 32 new records, written out coalesced
+  __shared__ float stage_s[256 / 32][32 * SMAX];   // each warp's 32 new records, written out coalesced
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   float* st = stage_s[warp];
   if (tid < ZD) z_s[tid] = C.z ? C.z[tid] : C.zin[tid];
@@ -523,7 +528,9 @@ __global__ void __launch_bounds__(256) cz_step(const CentralParams C) {
     NoiseGen gen{p, C.k, C.rk, u32x4{0u, 0u, b0.z, b0.w}};
     typename Model::Acc A;
     float* rec = st + lane * S;
-    if constexpr (Model::CHUNKED) {
+    if constexpr (RT) {
+      SampleRuntime<Model>::run(C.mc, C.nj, hsu_s, z_s, x, gen, A, [rec](int c, float v) { rec[c] = v; });
+    } else if constexpr (Model::CHUNKED) {
       SampleChunked<Model>::run(C.mc, hsu_s, z_s, x, gen, A, [rec](int c, float v) { rec[c] = v; });
     } else {
       SampleStream<Model, 0>::run(C.mc, hsu_s, z_s, x, gen, A, [rec](int c, float v) { rec[c] = v; });
@@ -614,7 +621,7 @@ cudaError_t central_step(int model, int nj, const CentralParams& c, int grid, cu
     case 2: return central_step_m<ArmPlanar<2>>(c, grid, s);
     case 5: return central_step_m<ArmPlanar<5>>(c, grid, s);
     case 28: return central_step_m<ArmPlanar<28>>(c, grid, s);
-    default: return cudaErrorInvalidValue;
+    default: return nj >= 1 && nj <= 28 ? central_step_m<ArmDyn<28>>(c, grid, s) : cudaErrorInvalidValue;
   }
 }
 
@@ -647,7 +654,9 @@ int central_grid(int model, int nj, int sms) {
       case 2: e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, cz_step<ArmPlanar<2>>, 256, 0); break;
       case 5: e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, cz_step<ArmPlanar<5>>, 256, 0); break;
       case 28: e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, cz_step<ArmPlanar<28>>, 256, 0); break;
-      default: break;
+      default:
+        if (nj >= 1 && nj <= 28) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, cz_step<ArmDyn<28>>, 256, 0);
+        break;
     }
   }
   return (e == cudaSuccess && bps > 0) ? bps * sms : 0;

@@ -20,6 +20,7 @@ struct CentralParams {
   const float* lw_in;       // [M] log-weights of step k-1
   float* lw_out;            // [M] log-weights of step k
   long long M;
+  int d, nj;                // state dimension and joints (read by runtime-dimension models only)
   unsigned long long* cl;   // [M] per-tile inclusive sums of q
   unsigned long long* tile_sum;    // [M / tile]
   unsigned long long* tile_incl;   // [M / tile] inclusive prefix of the tile sums

@@ -142,8 +142,7 @@ pf_status validate(const pf_config* cfg, const pf_model_params* mp, Geometry* g)
     if (cfg->resampler == PF_RESAMPLE_VOSE && m > pf::kCentralVoseMax) return PF_EUNSUPPORTED;
     if (cfg->resample_policy != PF_POLICY_ALWAYS) return PF_EUNSUPPORTED;
     g->vose = cfg->resampler == PF_RESAMPLE_VOSE;
-    if (g->model == PF_MODEL_ARM_PLANAR && g->nj != 2 && g->nj != 5 && g->nj != 28) return PF_EUNSUPPORTED;
-    g->m = m;
+    g->m = m;   // (any n_j <= 28: compiled 2 / 5 / 28, the generic arm otherwise)
     g->N = 1;
     g->deg = 0;
     g->tt = 1;
@@ -372,6 +371,8 @@ pf::CentralParams central_params(pf_handle* h, long long k) {
   c.lw_in = central_lw_of(h, c.in);
   c.lw_out = central_lw_of(h, c.out);
   c.M = h->g.M_local;
+  c.d = h->g.d;
+  c.nj = h->g.nj;
   u64* aux = reinterpret_cast<u64*>(h->parts + central_floats(h->g));
   c.cl = aux;
   c.tile_sum = aux + h->g.M_local;

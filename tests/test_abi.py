@@ -89,9 +89,9 @@ def test_unsupported_model(B):
     assert B.lib().pf_query_sizes(C.byref(_cfg(B)), C.byref(_model(B, 7)), C.byref(out)) == B.PF_OK
     assert out.state == 4 * (7 + 4 + 1) * 16 * 64
     assert B.lib().pf_query_sizes(C.byref(_cfg(B)), C.byref(_model(B, 29)), C.byref(out)) == B.PF_EUNSUPPORTED
-    # the centralized filter is compiled for n_j in {2, 5, 28} only
+    # the centralized filter too (the generic arm for n_j = 7)
     assert B.lib().pf_query_sizes(C.byref(_cfg(B, m=8192, n_filters=1, t=0, topo=0)), C.byref(_model(B, 7)),
-                                  C.byref(out)) == B.PF_EUNSUPPORTED
+                                  C.byref(out)) == B.PF_OK
     assert (5, 256) in B.pf_supported() and (28, 256) in B.pf_supported()
     assert B.pf_strerror(B.PF_EINVAL).startswith("invalid")
 

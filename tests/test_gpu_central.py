@@ -174,3 +174,24 @@ def test_central_resample_tables_bit_exact(P, orc, W, M, kind):
             ref = np.array([orc.rws_draw(q, int(a)) for a in ua], np.int32)
         np.testing.assert_array_equal(anc, ref)
         assert np.all(q[anc] > 0)   # never a zero-weight slot
+
+
+@pytest.mark.parametrize("nj,res", [(3, "rws"), (9, "vose")])
+def test_central_generic_arm(P, orc, W, nj, res):
+    # the centralized filter with the generic arm (n_j not compiled): a few
+    # steps bit for bit against the oracle, estimate every step
+    M = 8192
+    tr = W.make_trajectory(nj, 6, 4)
+    g = P.ParticleFilter(tr["mu0"], tr["sigma0"], P.ArmModel(n_joints=nj), m=M, n_filters=1, t=0, topo="none",
+                         resampler=res, seed=9)
+    o = orc.Filter(orc.Config(m=M, n_filters=1, t=0, topo="none", resampler=res, seed=9), orc.Model(n_joints=nj),
+                   tr["mu0"], tr["sigma0"])
+    for k in range(1, 6):
+        g.step(tr["Z"][k], tr["U"][k - 1])
+        o.step(tr["Z"][k], tr["U"][k - 1])
+        assert g.estimate()[2] == o.estimate()[2]
+    sg, wg, _ = g.get_particles()
+    so, wo, _ = o.get()
+    np.testing.assert_array_equal(sg, so)
+    np.testing.assert_array_equal(wg, wo)
+    g.close()
