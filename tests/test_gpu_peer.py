@@ -31,7 +31,8 @@ def P():
 @pytest.mark.timeout(120)
 @pytest.mark.parametrize("topo,N,world,t", [("ring", 16, 2, 1), ("ring", 8, 4, 1), ("torus", 64, 2, 1),
                                             ("torus", 16, 4, 1), ("ring", 4, 4, 1), ("all2all", 16, 2, 2),
-                                            ("all2all", 8, 4, 1), ("all2all", 32, 4, 3)])
+                                            ("all2all", 8, 4, 1), ("all2all", 32, 4, 3),
+                                            ("ring", 16, 8, 1), ("torus", 64, 8, 1), ("all2all", 16, 8, 2)])   # 8 ranks
 def test_peer_transport_local(P, orc, W, topo, N, world, t):
     import torch
     nj, m, T = 5, 64, 6
