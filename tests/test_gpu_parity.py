@@ -371,3 +371,26 @@ def test_device_inputs_streamed_and_batched(P, orc, W, central):
     np.testing.assert_array_equal(xb, xo)
     g.close()
     gb.close()
+
+
+@pytest.mark.parametrize("nj,m,N,t,topo,sig", [
+    (5, 32, 1, 1, "ring", 0.1),      # one sub-filter: its ring neighbours are itself (both sides)
+    (5, 32, 2, 3, "ring", 0.1),      # two sub-filters: both neighbours are the other one
+    (2, 64, 4, 1, "torus", 0.1),     # 2 x 2 torus: duplicate neighbours deliver the same particle twice
+    (2, 64, 8, 1, "ring", 0.0),      # zero process noise: deterministic motion, ties everywhere
+])
+def test_degenerate_filters(P, orc, W, nj, m, N, t, topo, sig):
+    tr = W.make_trajectory(nj, 8, 1)
+    gm = P.ArmModel(n_joints=nj, sigma_theta=sig, sigma_pos=sig, sigma_vel=sig)
+    om = orc.Model(n_joints=nj, sigma_theta=sig, sigma_pos=sig, sigma_vel=sig)
+    g = P.ParticleFilter(tr["mu0"], tr["sigma0"], gm, m=m, n_filters=N, t=t, topo=topo, seed=6)
+    o = orc.Filter(orc.Config(m=m, n_filters=N, t=t, topo=topo, seed=6), om, tr["mu0"], tr["sigma0"])
+    for k in range(1, 9):
+        g.step(tr["Z"][k], tr["U"][k - 1])
+        o.step(tr["Z"][k], tr["U"][k - 1])
+        assert g.estimate()[2] == o.estimate()[2]
+    sg, wg, _ = g.get_particles()
+    so, wo, _ = o.get()
+    np.testing.assert_array_equal(sg, so)
+    np.testing.assert_array_equal(wg, wo)
+    g.close()
