@@ -621,7 +621,9 @@ cudaError_t central_step(int model, int nj, const CentralParams& c, int grid, cu
     case 2: return central_step_m<ArmPlanar<2>>(c, grid, s);
     case 5: return central_step_m<ArmPlanar<5>>(c, grid, s);
     case 28: return central_step_m<ArmPlanar<28>>(c, grid, s);
-    default: return nj >= 1 && nj <= 28 ? central_step_m<ArmDyn<28>>(c, grid, s) : cudaErrorInvalidValue;
+    default:   // the generic arm, the smallest record stage that holds n_j
+      if (nj >= 1 && nj <= 8) return central_step_m<ArmDyn<8>>(c, grid, s);
+      return nj >= 1 && nj <= 28 ? central_step_m<ArmDyn<28>>(c, grid, s) : cudaErrorInvalidValue;
   }
 }
 
@@ -655,7 +657,9 @@ int central_grid(int model, int nj, int sms) {
       case 5: e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, cz_step<ArmPlanar<5>>, 256, 0); break;
       case 28: e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, cz_step<ArmPlanar<28>>, 256, 0); break;
       default:
-        if (nj >= 1 && nj <= 28) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, cz_step<ArmDyn<28>>, 256, 0);
+        if (nj >= 1 && nj <= 8) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, cz_step<ArmDyn<8>>, 256, 0);
+        else if (nj >= 1 && nj <= 28)
+          e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, cz_step<ArmDyn<28>>, 256, 0);
         break;
     }
   }

@@ -185,7 +185,7 @@ struct KCfg {
   static constexpr int ROW = (D + 1) * M;    // floats per sub-filter block
   static constexpr bool SCAN32 = (M <= 512);  // Q <= M 2^22 fits 32 bits
   static constexpr bool STAGED = UNR < P;    // rolled sample loop: per-slot values via smem
-  static constexpr bool X2 = X2_ && (P % 2 == 0) && !Model::RUNTIME;   // two particles at once (packed f32x2)
+  static constexpr bool X2 = X2_ && (P % 2 == 0);   // two particles at once (packed f32x2)
   static constexpr bool CHUNKED = Model::CHUNKED;   // runtime loop over joint chunks (pf_model.cuh)
   static_assert(P >= 1 && P * T == M, "M must be a multiple of the group size");
   static_assert(P <= 32, "exclusion masks are 32-bit");
@@ -756,6 +756,29 @@ struct SampleRuntime {
   }
 };
 
+template <class Model>
+struct SampleRuntime2 {
+  template <typename X, typename O>
+  __device__ __forceinline__ static void run(const ModelConsts2& mc, int nj, const f2* hsu2, const f2* z2, const X& x,
+                                             NoiseGen2& gen, typename Model::Acc2& A, const O& out) {
+    const int d = nj + 4;
+    u32x4 ba = gen.ba, bb = gen.bb;
+#pragma unroll 1
+    for (int q = 0; q < (d + 1) / 2; ++q) {
+      const int w = 2 + 2 * q;
+      if ((w & 3) == 0) {
+        ba = philox4x32_10_rk(gen.pa, gen.k, 0u, static_cast<uint32_t>(w >> 2), gen.rk);
+        bb = philox4x32_10_rk(gen.pb, gen.k, 0u, static_cast<uint32_t>(w >> 2), gen.rk);
+      }
+      const bool hi = (w & 3) == 2;
+      f2 z0, z1;
+      normal_pair2(hi ? ba.z : ba.x, hi ? ba.w : ba.y, hi ? bb.z : bb.x, hi ? bb.w : bb.y, z0, z1);
+      out(2 * q, Model::take_rt2(2 * q, nj, mc, hsu2, z2, x, z0, A));
+      if (2 * q + 1 < d) out(2 * q + 1, Model::take_rt2(2 * q + 1, nj, mc, hsu2, z2, x, z1, A));
+    }
+  }
+};
+
 // Peer transport, halo rows (reading R3/R4 and the halo plan of
 // distributed.py): ring — local sub-filter 0 -> the previous rank's row
 // n_local + 1, the last -> the next rank's row n_local; torus — the first grid
@@ -1321,7 +1344,9 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
           outa[c * M] = lo2(v);
           outb[c * M] = hi2(v);
         };
-        if constexpr (C::CHUNKED) {
+        if constexpr (RT) {
+          SampleRuntime2<Model>::run(P.mc2, P.nj, hsu2_s, z2_s, x, gen, A, store2);
+        } else if constexpr (C::CHUNKED) {
           SampleChunked2<Model>::run(P.mc2, hsu2_s, z2_s, x, gen, A, store2);
         } else {
           SampleStream2<Model, 0>::run(P.mc2, hsu2_s, z2_s, x, gen, A, store2);

@@ -176,11 +176,12 @@ struct ArmPlanar {
 // --------------------------------------------- the generic (runtime) arm ---
 // The arm for ANY n_joints <= NJMAX (the fallback behind the compiled
 // instances n_j in {2, 5, 28}): the same F8–F10 arithmetic in the same order
-// as ArmPlanar<n_j>, with the joint count a runtime value (take_rt, one
-// component at a time; SampleRuntime in pf_kernels.cuh pairs the normals),
-// so its results are bit-identical to a compiled instance of that n_j.  The
-// kernel's shared-memory stage is sized for NJMAX + 4 components; the HBM
-// block and mailbox entries use the runtime d.  One particle per thread.
+// as ArmPlanar<n_j>, with the joint count a runtime value (take_rt / take_rt2,
+// one component at a time; SampleRuntime(2) in pf_kernels.cuh pairs the
+// normals), so its results are bit-identical to a compiled instance of that
+// n_j.  The kernel's shared-memory stage is sized for NJMAX + 4 components
+// (instantiated for NJMAX = 8, 16, 28: the smallest bucket that holds n_j is
+// taken); the HBM block and mailbox entries use the runtime d.
 template <int NJMAX_>
 struct ArmDyn {
   static constexpr int kId = MODEL_ARM_PLANAR;
@@ -215,6 +216,32 @@ struct ArmDyn {
   }
   __device__ __forceinline__ static float finish(const ModelConsts& mc, const float* z, const Acc& A) {
     return ArmPlanar<1>::finish(mc, z, A);   // camera frame + residuals: independent of n_j
+  }
+  // the same on a pair of particles (packed, bit-identical lane by lane)
+  template <typename X>
+  __device__ __forceinline__ static f2 take_rt2(int c, int nj, const ModelConsts2& mc, const f2* hs_u2, const f2* z2,
+                                                const X& x, f2 xi, Acc2& A) {
+    if (c < nj) {
+      const f2 th = fma2(mc.s_th, xi, add2(x(c), hs_u2[c]));
+      A.phi = add2(A.phi, th);
+      sincos_c2(A.phi, A.s, A.c);
+      A.px = fma2(mc.lj, A.c, A.px);
+      A.py = fma2(mc.lj, A.s, A.py);
+      const f2 r = mul2(sub2(z2[2 + c], th), mc.inv_thm);
+      A.acc = (c == 0) ? mul2(r, r) : fma2(r, r, A.acc);
+      return th;
+    } else if (c == nj) {
+      A.xn = fma2(mc.s_pos, xi, fma2(mc.hs, x(nj + 2), x(nj)));
+      return A.xn;
+    } else if (c == nj + 1) {
+      A.yn = fma2(mc.s_pos, xi, fma2(mc.hs, x(nj + 3), x(nj + 1)));
+      return A.yn;
+    } else {
+      return fma2(mc.s_vel, xi, x(c));
+    }
+  }
+  __device__ __forceinline__ static f2 finish2(const ModelConsts2& mc, const f2* z2, const Acc2& A) {
+    return ArmPlanar<1>::finish2(mc, z2, A);
   }
 };
 

@@ -16,7 +16,7 @@ namespace pf {
 struct StepParams;
 
 struct KernelEntry {
-  int model, nj, m, res;          // pf_model_id; n_joints (arm; 0 = the generic arm) or 1
+  int model, nj, m, res;          // pf_model_id; n_joints (arm; -NJMAX = a generic bucket) or 1
   int gw, s, nstage, unr, minb;   // warps per group, groups per CTA, TMA stages, sample unroll, min CTAs/SM
   int large;                      // preferred when the shard has >= kLargeNLocal sub-filters
   cudaError_t (*prepare)(int* blocks_per_sm);
@@ -34,7 +34,7 @@ extern const KernelEntry kEntriesNJ28[];
 extern const int kNumEntriesNJ28;
 extern const KernelEntry kEntriesLG1[];
 extern const int kNumEntriesLG1;
-extern const KernelEntry kEntriesARMG[];   // the generic arm: n_joints key 0 = any n_j <= 28
+extern const KernelEntry kEntriesARMG[];   // the generic arm: n_joints key -NJMAX = any n_j <= NJMAX
 extern const int kNumEntriesARMG;
 }  // namespace pf
 

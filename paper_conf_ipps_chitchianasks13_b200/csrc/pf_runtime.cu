@@ -51,7 +51,9 @@ constexpr int kTables = 5;
 constexpr int kMaxGenericNJ = 28;   // the generic arm's stage holds d <= 32
 
 bool matches(const pf::KernelEntry& e, int model, int nj, int m, int res) {
-  return e.model == model && (model != PF_MODEL_ARM_PLANAR || e.nj == nj || e.nj == 0) && e.m == m && e.res == res;
+  // arm entries: a compiled n_j, or a generic bucket (key -NJMAX) that holds n_j
+  return e.model == model && (model != PF_MODEL_ARM_PLANAR || e.nj == nj || (e.nj < 0 && nj <= -e.nj)) && e.m == m &&
+         e.res == res;
 }
 
 // First entry matching (model, nj, m, res), or the PF_VARIANT-th one if set.
@@ -1202,7 +1204,7 @@ int32_t pf_supported(int32_t* n_joints, int32_t* m, int32_t cap) {
   for (int ti = 0; ti < kTables; ++ti) {
     const Table t = tables(ti);
     for (int i = 0; i < t.n; ++i) {
-      if (t.e[i].model != PF_MODEL_ARM_PLANAR || t.e[i].nj == 0) continue;
+      if (t.e[i].model != PF_MODEL_ARM_PLANAR || t.e[i].nj <= 0) continue;
       bool dup = false;
       for (int j = 0; j < i; ++j) dup = dup || (t.e[j].m == t.e[i].m && t.e[j].nj == t.e[i].nj);
       if (t.e[i].res != 0 || dup) continue;

@@ -48,9 +48,11 @@ if __name__ == "__main__":
         for topo in ["ring", "torus", "all2all"]:
             for t in [0, 1, 2, 4]:
                 run("t", 5, 256, 16384, topo=topo, t=t)
-    if "dim" in which:     # Fig.4c / C4: state dimension
+    if "dim" in which:     # Fig.4c / C4: state dimension (n_j = 2, 5, 28 compiled; the others the generic arm)
         for nj in [2, 5, 28]:
             run("dim", nj, 256, 65536)
+        for nj in [3, 7, 11, 16, 22]:
+            run("dim-generic", nj, 256, 65536)
     if "res" in which:     # Fig.5: RWS vs Vose
         for nj, N in [(5, 4096), (5, 65536), (28, 65536)]:
             for res in ["rws", "vose"]:
