@@ -555,12 +555,17 @@ __global__ void __launch_bounds__(256) cz_step(const CentralParams C) {
     const u64 v = warp_max_u64(lane < static_cast<int>(blockDim.x >> 5) ? red[lane] : 0ull);
     if (lane == 0) atomicMax(C.key_cur, v);
   }
-  __threadfence();
+  // the barrier orders every thread's writes (records, key) before thread 0's
+  // completion count, a gpu-scope acquire-release RMW (cumulative); the last
+  // CTA's acquire orders its reads below after every other CTA's release
   __syncthreads();
-  if (tid == 0) s_last = (atomicAdd(C.counter, 1u) == gridDim.x - 1) ? 1u : 0u;
+  if (tid == 0) {
+    unsigned int prev;
+    asm volatile("atom.acq_rel.gpu.global.add.u32 %0, [%1], 1;" : "=r"(prev) : "l"(C.counter) : "memory");
+    s_last = (prev == gridDim.x - 1) ? 1u : 0u;
+  }
   __syncthreads();
   if (s_last) {
-    __threadfence();
     const u64 key = __ldcg(C.key_cur);
     const uint32_t gidx = 0xFFFFFFFFu - static_cast<uint32_t>(key);
     float* outs[3] = {C.record, C.est_out, C.record_host};
@@ -579,10 +584,9 @@ __global__ void __launch_bounds__(256) cz_step(const CentralParams C) {
       *C.key_next = 0ull;
       *C.counter = 0u;
     }
-    if (C.record_host) {   // completion word polled by pf_estimate (after the record, system scope)
-      __threadfence_system();
-      __syncthreads();
-      if (tid == 0) *reinterpret_cast<volatile uint32_t*>(C.record_host + kRecordSeq) = C.k;
+    if (C.record_host) {   // completion word polled by pf_estimate: the barrier orders the
+      __syncthreads();     // record before thread 0's system-scope release (cumulative)
+      if (tid == 0) st_release_sys_u32(reinterpret_cast<uint32_t*>(C.record_host + kRecordSeq), C.k);
     }
   }
 }

@@ -1568,7 +1568,8 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
           for (int r = 0; r < P.world; ++r)
             for (int c = 0; c < 4; ++c) peer_rec(P.peer_blk[r], par, P.rank)[c] = r4[c];
         }
-        __threadfence_system();
+        // the barrier orders every thread's peer writes before the flag
+        // stores below, system-scope releases (cumulative)
         __syncthreads();
         // Rendezvous number rv (not the step number: flags only grow, also
         // across pf_set_particles).  Ordering: a rank writes the records /
@@ -1654,10 +1655,9 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
               for (int c = 0; c < 4; ++c) outs[o][c] = r[c];
         }
       }
-      if (P.record_host) {   // completion word polled by pf_estimate (after the record, system scope)
-        __threadfence_system();
-        __syncthreads();
-        if (tid == 0) *reinterpret_cast<volatile uint32_t*>(P.record_host + kRecordSeq) = P.k;
+      if (P.record_host) {   // completion word polled by pf_estimate: the barrier orders the
+        __syncthreads();     // record before thread 0's system-scope release (cumulative)
+        if (tid == 0) st_release_sys_u32(reinterpret_cast<uint32_t*>(P.record_host + kRecordSeq), P.k);
       }
     }
     if (tid == 0) {
