@@ -214,10 +214,12 @@ pf_status pf_step_batch(pf_handle* h, int32_t T, const float* zs, const float* u
 
 /* The global estimate of the last step: the particle with the highest
  * weight (PAPER.md:16 §IV; :20 §VI-D; R6).  Blocks until that record is on
- * the host: after a host-input pf_step of a single-rank filter the step kernel
- * streams it into mapped pinned host memory followed by the step number, and
- * this call polls that word (work queued after the step may still be
- * running); otherwise it synchronizes the stream and copies the record.
+ * the host: after a host-input pf_step of a single-rank filter (or of a
+ * peer-connected rank) the step kernel streams it into mapped pinned host
+ * memory as 64-bit words, each tagged with the step number, and this call
+ * polls them until every word carries this step (work queued after the step
+ * may still be running); otherwise it synchronizes the stream and copies the
+ * record.
  * Device errors of the step are reported either way.
  * x_hat: host float[d]; logw, idx (global particle index): host, nullable.
  * PF_ESTATE before the first step. */

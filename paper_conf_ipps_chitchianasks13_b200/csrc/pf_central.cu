@@ -568,25 +568,24 @@ __global__ void __launch_bounds__(256) cz_step(const CentralParams C) {
   if (s_last) {
     const u64 key = __ldcg(C.key_cur);
     const uint32_t gidx = 0xFFFFFFFFu - static_cast<uint32_t>(key);
-    float* outs[3] = {C.record, C.est_out, C.record_host};
+    float* outs[2] = {C.record, C.est_out};
     const float* src = C.publish ? C.in : C.out;
     if (tid < D) {
       const float v = __ldcg(src + static_cast<long long>(gidx) * S + tid);
-      for (int o = 0; o < 3; ++o)
+      for (int o = 0; o < 2; ++o)
         if (outs[o]) outs[o][4 + tid] = v;
+      if (C.record_host) put_tagged(C.record_host, 4 + tid, v, C.k);
     }
     if (tid == 0) {
       const float r[4] = {__uint_as_float(static_cast<uint32_t>(key)), __uint_as_float(static_cast<uint32_t>(key >> 32)),
                           unord_f32(static_cast<uint32_t>(key >> 32)), 0.0f};
-      for (int o = 0; o < 3; ++o)
+      for (int o = 0; o < 2; ++o)
         if (outs[o])
           for (int c = 0; c < 4; ++c) outs[o][c] = r[c];
+      if (C.record_host)
+        for (int c = 0; c < 4; ++c) put_tagged(C.record_host, c, r[c], C.k);
       *C.key_next = 0ull;
       *C.counter = 0u;
-    }
-    if (C.record_host) {   // completion word polled by pf_estimate: the barrier orders the
-      __syncthreads();     // record before thread 0's system-scope release (cumulative)
-      if (tid == 0) st_release_sys_u32(reinterpret_cast<uint32_t*>(C.record_host + kRecordSeq), C.k);
     }
   }
 }

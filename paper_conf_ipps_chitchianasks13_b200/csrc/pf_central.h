@@ -34,7 +34,7 @@ struct CentralParams {
   const float* record_prev;   // estimate record of step k-1 (its key gives l_max)
   float* record;
   float* est_out;
-  float* record_host;
+  unsigned long long* record_host;   // nullable: tagged words of the mapped host record (put_tagged)
   uint32_t rk[20];
   uint32_t k;
   int first;     // k == 1 (or the sample-only test hook): no resampling

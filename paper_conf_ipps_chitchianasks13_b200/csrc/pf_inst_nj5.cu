@@ -33,6 +33,7 @@ extern "C" int pf_debug_timeline(unsigned long long* out, long long cap, int res
     if (cudaMemcpyToSymbol(pf::pf_tl2, init2, sizeof(init2)) != cudaSuccess) return -3;
     return cudaMemcpyToSymbol(pf::pf_tl, &zero, sizeof(zero)) == cudaSuccess ? 0 : -3;
   }
+  if (cap == -2) return cudaMemcpyFromSymbol(out, pf::pf_tl3, sizeof(unsigned long long) * 3 * 4096) == cudaSuccess ? 0 : -3;
   if (cap < 0) return cudaMemcpyFromSymbol(out, pf::pf_tl2, sizeof(unsigned long long) * 4) == cudaSuccess ? 0 : -3;
   return cudaMemcpyFromSymbol(out, pf::pf_tl, sizeof(unsigned long long) * cap) == cudaSuccess ? 0 : -3;
 }

@@ -44,10 +44,11 @@ enum : int { TOPO_NONE = 0, TOPO_RING = 1, TOPO_TORUS = 2, TOPO_A2A = 3 };
 enum : int { RES_RWS = 0, RES_VOSE = 1 };
 enum : int { POLICY_ALWAYS = 0, POLICY_ESS = 1, POLICY_FREQ = 2 };
 
-// mapped host record: [0, 4 + d) the estimate record, [48, 48 + d) the weighted
-// mean, word kRecordSeq the step number of the last record written (pf_estimate
-// polls it instead of synchronizing the stream)
-constexpr int kRecordSeq = 127;
+// mapped host buffer (128 floats): u64 words [0, 4 + d) the estimate record of
+// the last step, each tagged with the step number (put_tagged; pf_estimate
+// polls them instead of synchronizing the stream), floats [kMeanHost,
+// kMeanHost + d) the weighted mean
+constexpr int kMeanHost = 80;
 
 // Peer transport (world > 1 on one node, NVLink/NVSwitch peer memory): every
 // rank's runtime owns a small "peer block" that the other ranks write into:
@@ -78,7 +79,7 @@ struct StepParams {
   unsigned int* work;      // dynamic sub-filter counter (0 on entry, reset by the last CTA)
   float* record;           // [4 + d] estimate record of this shard
   float* est_out;          // nullable [4 + d] (batched mode)
-  float* record_host;      // nullable [4 + d]: mapped pinned host copy of the record
+  u64* record_host;        // nullable [4 + d]: mapped pinned host copy of the record (tagged words)
   long long* dbg_src;      // nullable [M_local] exchange sources (global index)
   int* dbg_anc;            // nullable [M_local] ancestors
   long long n_local, g0, n_global, R, C;
@@ -151,6 +152,7 @@ __device__ __forceinline__ void mbar_wait(u64* bar, uint32_t parity) {
 // dev-only timeline (scripts/timeline.py): one record of 8 u64 per sub-filter
 __device__ unsigned long long pf_tl[1 + 8 * 65536];
 __device__ unsigned long long pf_tl2[4];   // min CTA entry, last-CTA epilogue start, its end
+__device__ unsigned long long pf_tl3[3 * 4096];   // per CTA: entry, after griddepcontrol.wait, after the prologue
 __device__ __forceinline__ unsigned long long tl_now() {
   unsigned long long t;
   asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
@@ -934,7 +936,8 @@ static __device__ void pool_top_t(const StepParams& P, const float* mb, long lon
 template <class C>
 __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __grid_constant__ StepParams P) {
 #ifdef PF_TIMELINE
-  if (threadIdx.x == 0) atomicMin(&pf_tl2[0], tl_now());
+  const unsigned long long tl_entry = tl_now();
+  if (threadIdx.x == 0) atomicMin(&pf_tl2[0], tl_entry);
 #endif
   using Model = typename C::Model;
   constexpr int M = C::M, GW = C::GW, PP = C::P;
@@ -1010,6 +1013,9 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
   // step's tail; nothing that step wrote (particle blocks, mailbox, counters,
   // key, device inputs) is read before its grid has completed (no-op otherwise)
   asm volatile("griddepcontrol.wait;" ::: "memory");
+#ifdef PF_TIMELINE
+  const unsigned long long tl_pw = tl_now();
+#endif
   if (G.t == 0) {
     mbar_init(bars, 1);
     mbar_init(bars + 1, 1);
@@ -1032,6 +1038,13 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
   __syncthreads();
 
   TL(tl_start);
+#ifdef PF_TIMELINE
+  if (threadIdx.x == 0 && blockIdx.x < 4096) {
+    pf_tl3[3 * blockIdx.x] = tl_entry;
+    pf_tl3[3 * blockIdx.x + 1] = tl_pw;
+    pf_tl3[3 * blockIdx.x + 2] = tl_start;
+  }
+#endif
   for (int it = 0;; ++it) {
     const int st = (C::NSTAGE == 2) ? (it & 1) : 0;
     TL(tl_w0);
@@ -1041,13 +1054,6 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
     if (n >= P.n_local) break;
     if constexpr (C::NSTAGE == 2) {   // prefetch the next sub-filter into the other stage
       if (G.t == 0) issue(st ^ 1, fetch_next());
-    } else {
-      // one stage: the next sub-filter's block is loaded only after this one's
-      // sample loop; pull it from HBM into L2 now, so that load hits L2
-      if (G.t == 0) {
-        const long long nn = gstride + pending;
-        if (nn < P.n_local) bulk_prefetch_l2(P.parts + nn * ROW, stage_bytes);
-      }
     }
     float* xs = reinterpret_cast<float*>(gs + C::g_stage + st * C::stage_bytes);
     float* ws = xs + D * M;
@@ -1294,6 +1300,17 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
     }
 
     TL(tl_res);
+    if constexpr (C::NSTAGE == 1) {
+      // one stage: the next sub-filter's block is loaded only after this one's
+      // sample loop; pull it from HBM into L2 now, so that load hits L2.  Not
+      // earlier: the index is the ticket thread 0 requested a sub-filter ago,
+      // and the first one (the launch's burst of same-address atomics, one per
+      // group) returns only microseconds into the launch.
+      if (G.t == 0 && mode == MODE_STEP) {
+        const long long nn = gstride + pending;
+        if (nn < P.n_local) bulk_prefetch_l2(P.parts + nn * ROW, stage_bytes);
+      }
+    }
     if constexpr (C::X2) {
      if (do_sample) {
       // ---- a9 gather (smem) + a1 RNG + a2 sample + a3 weight + a10 store,
@@ -1538,7 +1555,7 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
       const uint32_t gidx = 0xFFFFFFFFu - static_cast<uint32_t>(key);
       const long long col = static_cast<long long>(gidx) - P.g0 * M;
       const float* blk = P.parts + (col / M) * ROW + (col % M);
-      float* outs[3] = {P.record, P.est_out, P.record_host};
+      float* outs[2] = {P.record, P.est_out};
       if (P.peer_mb[0] && (mode == MODE_STEP || mode == MODE_PUBLISH)) {
         // peer transport: the boundary sub-filters' best-t rows into the
         // neighbour ranks' halo rows, this shard's best record into slot
@@ -1608,8 +1625,9 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
           for (int c = tid; c < 4 + D; c += 32) {
             const float v = c == 3 ? __uint_as_float(timed_out ? kStatusPeerTimeout : 0u)
                                    : __ldcv(rec0 + src * kPeerRec + c);
-            for (int o = 0; o < 3; ++o)
+            for (int o = 0; o < 2; ++o)
               if (outs[o]) outs[o][c] = v;
+            if (P.record_host) put_tagged(P.record_host, c, v, static_cast<uint32_t>(P.k));
           }
           if (a2a) {   // the global pool: best t of the world's pool rows (pf_reduce_pool, fused)
             float* out = P.mb_cur + P.pool_row * P.tt * E;
@@ -1642,22 +1660,22 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
         if (tid < D) {
           const float v = __ldcg(blk + tid * M);
 #pragma unroll
-          for (int o = 0; o < 3; ++o)
+          for (int o = 0; o < 2; ++o)
             if (outs[o]) outs[o][4 + tid] = v;
+          if (P.record_host) put_tagged(P.record_host, 4 + tid, v, static_cast<uint32_t>(P.k));
         }
         if (tid == 0) {
           const float r[4] = {__uint_as_float(static_cast<uint32_t>(key)), __uint_as_float(static_cast<uint32_t>(key >> 32)),
                               unord_f32(static_cast<uint32_t>(key >> 32)), 0.0f};
 #pragma unroll
-          for (int o = 0; o < 3; ++o)
+          for (int o = 0; o < 2; ++o)
             if (outs[o])
 #pragma unroll
               for (int c = 0; c < 4; ++c) outs[o][c] = r[c];
+          if (P.record_host)
+#pragma unroll
+            for (int c = 0; c < 4; ++c) put_tagged(P.record_host, c, r[c], static_cast<uint32_t>(P.k));
         }
-      }
-      if (P.record_host) {   // completion word polled by pf_estimate: the barrier orders the
-        __syncthreads();     // record before thread 0's system-scope release (cumulative)
-        if (tid == 0) st_release_sys_u32(reinterpret_cast<uint32_t*>(P.record_host + kRecordSeq), P.k);
       }
     }
     if (tid == 0) {

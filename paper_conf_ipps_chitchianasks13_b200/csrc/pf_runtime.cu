@@ -289,7 +289,7 @@ pf::StepParams base_params(pf_handle* h, long long k, int mode) {
   p.counter = reinterpret_cast<unsigned int*>(h->scratch + kOffCounter);
   p.work = reinterpret_cast<unsigned int*>(h->scratch + kOffWork);
   p.record = record(h);
-  p.record_host = streams_record(h) ? h->rec_host_dev : nullptr;
+  p.record_host = streams_record(h) ? reinterpret_cast<u64*>(h->rec_host_dev) : nullptr;
   p.est_out = nullptr;
   p.dbg_src = nullptr;
   p.dbg_anc = nullptr;
@@ -400,7 +400,7 @@ pf::CentralParams central_params(pf_handle* h, long long k) {
   c.counter = reinterpret_cast<unsigned int*>(h->scratch + kOffCounter);
   c.record_prev = record(h);
   c.record = record(h);
-  c.record_host = streams_record(h) ? h->rec_host_dev : nullptr;
+  c.record_host = streams_record(h) ? reinterpret_cast<u64*>(h->rec_host_dev) : nullptr;
   const uint32_t key0 = static_cast<uint32_t>(h->cfg.seed), key1 = static_cast<uint32_t>(h->cfg.seed >> 32);
   for (int r = 0; r < 10; ++r) {
     c.rk[2 * r] = key0 + static_cast<uint32_t>(r) * 0x9E3779B9u;
@@ -597,7 +597,8 @@ pf_status pf_init(const pf_config* cfg, const pf_model_params* model, const pf_b
     h->peer_timeout_ns = static_cast<unsigned long long>(ms > 0 ? ms : 30000) * 1000000ull;
     h->pdl = std::getenv("PF_NO_PDL") == nullptr;
     h->last_mapped = false;
-    reinterpret_cast<volatile uint32_t*>(h->rec_host)[pf::kRecordSeq] = 0xFFFFFFFFu;
+    for (int c = 0; c < 4 + 32; ++c)   // no step's tag
+      reinterpret_cast<volatile uint64_t*>(h->rec_host)[c] = 0xFFFFFFFF00000000ull;
   }
   if (e != cudaSuccess) {
     pf_destroy(h);
@@ -738,35 +739,46 @@ pf_status pf_estimate(pf_handle* h, float* x_hat, float* logw, int64_t* idx) {
   if (h->err != PF_OK) return h->err;
   if (h->step < 1) return PF_ESTATE;
   // Host-input steps (the streaming, real-time use): the kernel wrote the
-  // record into mapped pinned host memory followed by the step number (system-
-  // scope fence in between), so waiting is polling that word — no stream
-  // synchronization on the critical path; a stream that completes without
-  // it (or any error) ends the poll.  Otherwise (device inputs, several
-  // ranks) the record is copied from the device after a stream synchronization.
+  // record into mapped pinned host memory as 64-bit words tagged with the
+  // step number, so waiting is polling those words until every one carries
+  // this step — no stream synchronization, and no fence in the kernel, on the
+  // critical path; a stream that completes without them (or any error) ends
+  // the poll.  Otherwise (device inputs, several ranks over NCCL) the record
+  // is copied from the device after a stream synchronization.
   cudaError_t e = cudaSuccess;
+  float rec[4 + 32 + 4];
+  const int nw = 4 + h->g.d;
   if (h->last_mapped) {
     const uint32_t want = static_cast<uint32_t>(h->step);
-    // acquire: the record loads below may not be reordered before the step
-    // number (the kernel wrote the record first, then a system-scope fence)
-    const uint32_t* seq = reinterpret_cast<const uint32_t*>(h->rec_host + pf::kRecordSeq);
-    for (unsigned it = 1; __atomic_load_n(seq, __ATOMIC_ACQUIRE) != want; ++it) {
-      if ((it & 1023u) == 0u) {
-        e = cudaStreamQuery(h->stream);
-        if (e != cudaErrorNotReady) break;
+    const uint64_t* words = reinterpret_cast<const uint64_t*>(h->rec_host);
+    auto tag = [](uint64_t w) { return static_cast<uint32_t>(w >> 32); };
+    unsigned it = 1;
+    for (int c = 0; c < nw && e == cudaSuccess; ++c) {
+      // each word is single-copy atomic: its value half belongs to its tag
+      uint64_t w = __atomic_load_n(words + c, __ATOMIC_ACQUIRE);
+      while (tag(w) != want) {
+        if ((it++ & 1023u) == 0u) {
+          const cudaError_t q = cudaStreamQuery(h->stream);
+          if (q != cudaErrorNotReady) {   // the stream is idle or failed: the word is final
+            w = __atomic_load_n(words + c, __ATOMIC_ACQUIRE);
+            if (q != cudaSuccess) e = q;
+            else if (tag(w) != want) e = cudaErrorUnknown;   // completed without this step's record
+            break;
+          }
+        }
+        w = __atomic_load_n(words + c, __ATOMIC_ACQUIRE);
       }
+      const uint32_t v = static_cast<uint32_t>(w);
+      std::memcpy(&rec[c], &v, 4);
     }
-    // the step number arrived after the record (system-scope fence): the
-    // record is complete.  A device error ends the poll through the query
-    // above; one raised after the record surfaces at the next call (sticky).
-    if (e == cudaErrorNotReady) e = cudaSuccess;
+    // an error raised after the record surfaces at the next call (sticky)
     if (e != cudaSuccess) return sticky(h, e);
   } else {
-    e = cudaMemcpyAsync(h->rec_host, record(h), sizeof(float) * (4 + h->g.d), cudaMemcpyDeviceToHost, h->stream);
+    e = cudaMemcpyAsync(h->rec_host, record(h), sizeof(float) * nw, cudaMemcpyDeviceToHost, h->stream);
     if (e == cudaSuccess) e = cudaStreamSynchronize(h->stream);
     if (e != cudaSuccess) return sticky(h, e);
+    std::memcpy(rec, const_cast<const float*>(h->rec_host), sizeof(float) * nw);
   }
-  float rec[4 + 32 + 4];
-  std::memcpy(rec, const_cast<const float*>(h->rec_host), sizeof(float) * (4 + h->g.d));
   uint32_t lo, status;
   std::memcpy(&lo, &rec[0], 4);
   std::memcpy(&status, &rec[3], 4);
@@ -804,12 +816,12 @@ pf_status pf_estimate_mean(pf_handle* h, float* x_mean) {
   if (h->cfg.world != 1) return PF_ESTATE;
   pf_status st = mean_partials_launch(h);
   if (st != PF_OK) return st;
-  float* out = h->rec_host_dev + 48;   // mapped pinned host floats [48, 48 + d) (record uses [0, 4 + d))
+  float* out = h->rec_host_dev + pf::kMeanHost;   // mapped pinned host floats (the record's tagged words are below)
   st = sticky(h, pf::mean_final(mean_scratch(h), pf::kMeanGrid, h->g.d, nullptr, nullptr, out, h->stream));
   if (st != PF_OK) return st;
   cudaError_t e = cudaStreamSynchronize(h->stream);
   if (e != cudaSuccess) return sticky(h, e);
-  std::memcpy(x_mean, const_cast<const float*>(h->rec_host) + 48, sizeof(float) * h->g.d);
+  std::memcpy(x_mean, const_cast<const float*>(h->rec_host) + pf::kMeanHost, sizeof(float) * h->g.d);
   return PF_OK;
 }
 
@@ -829,12 +841,12 @@ pf_status pf_mean_partial(pf_handle* h, double** partial_dev, int32_t* partial_d
 pf_status pf_reduce_means(pf_handle* h, const double* partials_dev, int32_t count, float* x_mean) {
   if (!h || !partials_dev || count < 1 || !x_mean) return PF_EINVAL;
   if (h->err != PF_OK) return h->err;
-  float* out = h->rec_host_dev + 48;
+  float* out = h->rec_host_dev + pf::kMeanHost;
   pf_status st = sticky(h, pf::mean_final(partials_dev, count, h->g.d, nullptr, nullptr, out, h->stream));
   if (st != PF_OK) return st;
   cudaError_t e = cudaStreamSynchronize(h->stream);
   if (e != cudaSuccess) return sticky(h, e);
-  std::memcpy(x_mean, const_cast<const float*>(h->rec_host) + 48, sizeof(float) * h->g.d);
+  std::memcpy(x_mean, const_cast<const float*>(h->rec_host) + pf::kMeanHost, sizeof(float) * h->g.d);
   return PF_OK;
 }
 
@@ -848,7 +860,7 @@ pf_status pf_record_ptr(pf_handle* h, float** record_dev, int32_t* record_floats
 pf_status pf_reduce_records(pf_handle* h, const float* records_dev, int32_t count) {
   if (!h || !records_dev || count < 1) return PF_EINVAL;
   if (h->err != PF_OK) return h->err;
-  pf_reduce_records_kernel<<<1, 32, 0, h->stream>>>(records_dev, count, 4 + h->g.d, record(h), h->rec_host_dev);
+  pf_reduce_records_kernel<<<1, 32, 0, h->stream>>>(records_dev, count, 4 + h->g.d, record(h), nullptr);
   return sticky(h, cudaGetLastError());
 }
 

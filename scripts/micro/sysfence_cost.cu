@@ -16,6 +16,13 @@ __global__ void pub_k(float* rec, unsigned* seq, unsigned k) {
     __syncthreads();
     if (tid == 0) asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(seq), "r"(k) : "memory");
   }
+  if (V == 6) {   // 13 words, each with the sequence number in its upper half (no fence)
+    if (tid < 13) {
+      const unsigned long long w = (static_cast<unsigned long long>(k) << 32) | __float_as_uint(static_cast<float>(k + tid));
+      asm volatile("st.relaxed.sys.global.u64 [%0], %1;" ::"l"(reinterpret_cast<unsigned long long*>(seq) + 8 + tid), "l"(w) : "memory");
+    }
+    return;
+  }
   if (V == 5) {
     __syncthreads();
     if (tid == 0) { __threadfence_system(); *(volatile unsigned*)seq = k; }
@@ -40,7 +47,13 @@ void run(const char* name, float* rec, unsigned* seq_d, volatile unsigned* seq_h
     for (int i = 0; i < R; ++i) {
       const unsigned want = k++;
       pub_k<V><<<1, 256, 0, s>>>(rec, seq_d, want);
-      while (__atomic_load_n(seq_h, __ATOMIC_ACQUIRE) != want) {}
+      if (V == 6) {
+        const unsigned long long* w = reinterpret_cast<const unsigned long long*>(const_cast<unsigned*>(seq_h)) + 8;
+        for (int j = 0; j < 13; ++j)
+          while ((__atomic_load_n(w + j, __ATOMIC_RELAXED) >> 32) != want) {}
+      } else {
+        while (__atomic_load_n(seq_h, __ATOMIC_ACQUIRE) != want) {}
+      }
     }
     rt = std::chrono::duration<double, std::micro>(clk::now() - a).count() / R;
     cudaStreamSynchronize(s);
@@ -51,7 +64,7 @@ int main() {
   cudaStream_t s; cudaStreamCreate(&s);
   float *rh, *rd, *dev; unsigned *sh, *sd;
   cudaHostAlloc(&rh, 256, cudaHostAllocMapped); cudaHostGetDevicePointer(&rd, rh, 0);
-  cudaHostAlloc(&sh, 64, cudaHostAllocMapped); cudaHostGetDevicePointer(&sd, sh, 0);
+  cudaHostAlloc(&sh, 256, cudaHostAllocMapped); cudaHostGetDevicePointer(&sd, sh, 0);
   cudaMalloc(&dev, 256);
   run<0>("record -> device memory", dev, sd, nullptr, s);
   run<0>("record -> host memory", rd, sd, nullptr, s);
@@ -61,6 +74,7 @@ int main() {
     run<3>("host, writers fence.sc.sys", rd, sd, sh, s);
     run<4>("host, bar + st.release.sys", rd, sd, sh, s);
     run<5>("host, bar + tid0 fence.sc.sys", rd, sd, sh, s);
+    run<6>("host, 13 x u64 {word, seq}, no fence", rd, sd, sh, s);
   }
   return 0;
 }

@@ -9,16 +9,17 @@ from paper_conf_ipps_chitchianasks13_b200 import binding, filter as F, workload 
 
 nj, m, N, res = int(sys.argv[1]), int(sys.argv[2]), int(sys.argv[3]), sys.argv[4]
 flush_l2 = len(sys.argv) <= 5 or sys.argv[5] != "0"
+host_in = len(sys.argv) > 6 and sys.argv[6] == "host"   # z / u through the launch (the e2e path)
 tr = W.make_trajectory(nj, 20, 0)
 g = F.ParticleFilter(tr["mu0"], tr["sigma0"], F.ArmModel(n_joints=nj), m=m, n_filters=N, resampler=res,
-                     device_inputs=True)
+                     device_inputs=not host_in)
 zs = torch.tensor(tr["Z"][1:], device="cuda"); us = torch.tensor(tr["U"][:-1], device="cuda")
 L = binding.lib()
 fn = L.pf_debug_timeline
 fn.argtypes = [C.c_void_p, C.c_longlong, C.c_int]
 flush = torch.empty(512 << 20, dtype=torch.uint8, device="cuda")
 for k in range(5):
-    g.step(zs[k], us[k])
+    g.step(*((tr["Z"][k + 1], tr["U"][k]) if host_in else (zs[k], us[k])))
 torch.cuda.synchronize()
 for rep in range(3):
     if flush_l2:
@@ -26,13 +27,26 @@ for rep in range(3):
     torch.cuda.synchronize()
     fn(None, 0, 1)
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    e0.record(g.stream); g.step(zs[5 + rep], us[5 + rep]); e1.record(g.stream)
+    if host_in:
+        zh, uh = tr["Z"][6 + rep], tr["U"][5 + rep]
+        e0.record(g.stream); g.step(zh, uh); e1.record(g.stream)
+    else:
+        e0.record(g.stream); g.step(zs[5 + rep], us[5 + rep]); e1.record(g.stream)
     torch.cuda.synchronize()
     buf = np.zeros(1 + 8 * 65536, np.uint64)
     fn(buf.ctypes.data, buf.size, 0)
     t2 = np.zeros(4, np.uint64)
     fn(t2.ctypes.data, -1, 0)
     n = int(buf[0]); r = buf[1:1 + 8 * n].reshape(n, 8).astype(np.int64)
+    t3 = np.zeros(3 * 4096, np.uint64)
+    fn(t3.ctypes.data, -2, 0)
+    t3 = t3.reshape(4096, 3).astype(np.int64)
+    t3 = t3[t3[:, 0] > 0]
+    if len(t3):   # per-CTA prologue: entry -> after griddepcontrol.wait -> after the prologue barrier
+        e0_ = t3[:, 0].min()
+        q = lambda v: f"p50 {np.median(v)/1e3:.2f} p90 {np.percentile(v, 90)/1e3:.2f} max {v.max()/1e3:.2f}"
+        print(f"  CTAs {len(t3)}: entry (from first) {q(t3[:, 0] - e0_)}; wait {q(t3[:, 1] - t3[:, 0])}; "
+              f"prologue {q(t3[:, 2] - t3[:, 1])}; ready-to-loop (from first entry) {q(t3[:, 2] - e0_)}")
     tmin = int(r[:, 1].min())
     print(f"  first CTA entry -> first group start {(tmin - int(t2[0]))/1e3:.2f} us; last group end -> "
           f"epilogue (last CTA) start {(int(t2[1]) - int(r[:, 7].max()))/1e3:.2f} us; epilogue {(int(t2[2]) - int(t2[1]))/1e3:.2f} us")
