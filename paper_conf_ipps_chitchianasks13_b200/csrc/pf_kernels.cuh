@@ -135,6 +135,16 @@ __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t by
 __device__ __forceinline__ void bulk_prefetch_l2(const void* src, uint32_t bytes) {
   asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(src), "r"(bytes) : "memory");
 }
+// relaxed fetch-and-add of 1 on the launch's work counter, not aggregated
+// across the warp: the result register is consumed only where it is used
+__device__ __forceinline__ unsigned int ticket_add(unsigned int* p) {
+  unsigned int r;
+  // atom.inc with a limit the counter never reaches is an add of 1 that ptxas
+  // does not aggregate (it rewrites atom.add, and inc with limit 2^32-1, into
+  // a warp-aggregated atomic + shuffle)
+  asm volatile("atom.relaxed.gpu.global.inc.u32 %0, [%1], 0x7FFFFFFF;" : "=r"(r) : "l"(p));
+  return r;
+}
 __device__ __forceinline__ void mbar_arrive(u64* bar) {
   asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
 }
@@ -1001,11 +1011,16 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
     }
   };
   // thread 0 keeps one dynamic index in flight: the atomic's latency is
-  // hidden behind a whole sub-filter of work
+  // hidden behind a whole sub-filter of work.  The ticket is taken with a
+  // plain PTX atom: atomicAdd() is compiled into a warp-aggregated atomic
+  // whose result is shuffled to the lanes at once, i.e. consumed right away,
+  // which stalled thread 0's warp (and at the next barrier its group) for the
+  // atomic's round trip on every sub-filter, and the launch's prologue for
+  // the burst of same-address atomics of all groups (~4 us at C2).
   unsigned int pending = 0;
   auto fetch_next = [&]() -> long long {
     const long long nn = gstride + pending;
-    pending = atomicAdd(P.work, 1u);
+    pending = ticket_add(P.work);
     return nn;
   };
 
@@ -1021,7 +1036,7 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
     mbar_init(bars + 1, 1);
     fence_mbar_init();
     issue(0, gid0);
-    if (gid0 < P.n_local) pending = atomicAdd(P.work, 1u);
+    if (gid0 < P.n_local) pending = ticket_add(P.work);
   }
   if (do_sample) {
     if (threadIdx.x < ZD) {
