@@ -442,72 +442,143 @@ __device__ __forceinline__ void resample_group(const uint32_t (&q)[C::P], const 
     // Vose's alias method (PAPER.md:18 §IV, :20–22 §VI-F), table by the
     // closed form of the sequential sweep (R10): a_j = M q_j, small L =
     // {a < Q}, D = inclusive deficits over L, E = inclusive excesses over H.
-    // Two slot-order scans: the weights (-> Q and the prefix of a = M q), and
+    // Two slot-order prefix sums: the weights (-> the prefix of a = M q), and
     // the deficits over L with the count of L packed above bit 48 (D < 2^42).
     // E follows from sum_{j'<=j} (a_j' - Q) = E_j - D_j.
-    // Only the two inclusive scans stay live per slot (register budget); the
-    // per-slot class, deficit, counts and E are recomputed from them.
-    u64 qinc[P], pinc[P];
-    u64 Qg, ptot;
-    if constexpr (C::SCAN32) {   // Q <= M 2^22 fits 32 bits: the weight scan in u32
-      uint32_t val[P];
+    u64 Qg, Dtot;
+    int nL;
+    if constexpr (C::SCAN32) {
+      // Q <= M 2^22 fits 32 bits.  Q first (warp REDUX + one group barrier),
+      // then ONE transposition of q into slot order: thread t classifies its
+      // CONTIGUOUS slots [tP, tP + P) itself and scans, in registers, both the
+      // weights (u32) and the packed deficits (u64) — one warp scan level and
+      // one cross-warp level for the two — and writes its list entries
+      // straight from registers (no scan results stored back to shared memory
+      // and re-read).  5 group barriers per table instead of 8; the same
+      // sums, hence the same table.
+      uint32_t qs = 0;
 #pragma unroll
-      for (int j = 0; j < P; ++j) val[j] = q[j];
-      uint32_t* b32 = reinterpret_cast<uint32_t*>(S.scan);
-      Qg = slot_scan_smem<C, uint32_t>(val, b32, G);
+      for (int j = 0; j < P; ++j) qs += q[j];
+      qs = __reduce_add_sync(0xFFFFFFFFu, qs);
+      if constexpr (C::GW > 1) {
+        uint32_t* r = reinterpret_cast<uint32_t*>(G.red + G.rb * 32);
+        G.rb ^= 1;
+        if (G.lane == 0) r[G.wig] = qs;
+        uint32_t* b32 = reinterpret_cast<uint32_t*>(S.scan);
 #pragma unroll
-      for (int j = 0; j < P; ++j) qinc[j] = b32[C::slot(G.t, j)];
-    } else {
-      u64 val[P];
+        for (int j = 0; j < P; ++j) b32[C::slot(G.t, j)] = q[j];
+        gsync<C::GW>(G.g);
+        qs = 0;
 #pragma unroll
-      for (int j = 0; j < P; ++j) val[j] = q[j];
-      Qg = slot_scan_smem<C, u64>(val, S.scan, G);
+        for (int w = 0; w < C::GW; ++w) qs += r[w];
+      } else {
+        uint32_t* b32 = reinterpret_cast<uint32_t*>(S.scan);
 #pragma unroll
-      for (int j = 0; j < P; ++j) qinc[j] = S.scan[C::slot(G.t, j)];
-    }
-    {
-      u64 packed[P];
+        for (int j = 0; j < P; ++j) b32[C::slot(G.t, j)] = q[j];
+        __syncwarp();
+      }
+      const uint32_t Q32 = qs;
+      Qg = Q32;
+      uint32_t qc[P], qi[P];   // contiguous slots tP + e: weight, inclusive weight sum
+      u64 pc[P];               // packed inclusive deficit sum (count of L above bit 48)
+      vload<uint32_t, P>(reinterpret_cast<const uint32_t*>(S.scan) + G.t * P, qc);
+#pragma unroll
+      for (int e = 0; e < P; ++e) {
+        const u64 a = static_cast<u64>(M) * qc[e];
+        const u64 pk0 = a < Qg ? (Qg - a) + (1ull << 48) : 0ull;
+        qi[e] = e ? qi[e - 1] + qc[e] : qc[e];
+        pc[e] = e ? pc[e - 1] + pk0 : pk0;
+      }
+      const uint32_t tq = qi[P - 1];
+      const u64 tp = pc[P - 1];
+      const uint32_t iq = warp_incl_scan<uint32_t>(tq, G.lane);
+      const u64 ip = warp_incl_scan<u64>(tp, G.lane);
+      uint32_t oq = iq - tq;
+      u64 op = ip - tp, ptot;
+      if constexpr (C::GW == 1) {
+        ptot = __shfl_sync(0xFFFFFFFFu, ip, 31);
+      } else {
+        u64* r = G.red + G.rb * 32;
+        G.rb ^= 1;
+        if (G.lane == 31) {
+          r[G.wig] = ip;
+          r[16 + G.wig] = iq;
+        }
+        gsync<C::GW>(G.g);
+        ptot = 0;
+#pragma unroll
+        for (int w = 0; w < C::GW; ++w) {
+          const u64 xp = r[w];
+          if (w < G.wig) {
+            op += xp;
+            oq += static_cast<uint32_t>(r[16 + w]);
+          }
+          ptot += xp;
+        }
+      }
+      nL = static_cast<int>(ptot >> 48);
+      Dtot = ptot & ((1ull << 48) - 1);
+      // (every thread's transposition reads precede the barrier above, so the
+      // lists may now overwrite S.scan)
+#pragma unroll
+      for (int e = 0; e < P; ++e) {
+        const int s = G.t * P + e;
+        const u64 a = static_cast<u64>(M) * qc[e];
+        const bool small = a < Qg;
+        const u64 pinc = pc[e] + op;
+        const u64 Dinc = pinc & ((1ull << 48) - 1);
+        const int ls = static_cast<int>(pinc >> 48) - (small ? 1 : 0);   // smalls before the slot
+        if (small) {
+          S.lists[ls] = s;
+          S.scan[ls] = Dinc - (Qg - a);
+        } else {   // E_s = D_s + sum_{s' <= s} (a_s' - Q): 32 x 32 -> 64-bit products
+          S.lists[nL + (s - ls)] = s;
+          S.scan[nL + (s - ls)] = Dinc + static_cast<u64>(qi[e] + oq) * static_cast<uint32_t>(M) -
+                                  static_cast<u64>(static_cast<uint32_t>(s) + 1u) * Q32;
+        }
+      }
+    } else {   // m = 1024: Q up to 2^32, both scans in u64 through shared memory
+      u64 qinc[P], pinc[P];
+      u64 ptot;
+      {
+        u64 val[P];
+#pragma unroll
+        for (int j = 0; j < P; ++j) val[j] = q[j];
+        Qg = slot_scan_smem<C, u64>(val, S.scan, G);
+#pragma unroll
+        for (int j = 0; j < P; ++j) qinc[j] = S.scan[C::slot(G.t, j)];
+      }
+      {
+        u64 packed[P];
+#pragma unroll
+        for (int j = 0; j < P; ++j) {
+          const u64 a = static_cast<u64>(M) * q[j];
+          packed[j] = a < Qg ? (Qg - a) + (1ull << 48) : 0ull;
+        }
+        ptot = slot_scan_smem<C, u64>(packed, S.prob, G);
+#pragma unroll
+        for (int j = 0; j < P; ++j) pinc[j] = S.prob[C::slot(G.t, j)];
+      }
+      // (every thread read qinc before passing scan 2's barriers: S.scan is free)
+      nL = static_cast<int>(ptot >> 48);
+      Dtot = ptot & ((1ull << 48) - 1);
+      // Lists: small slots ascending with their EXCLUSIVE deficit sums A_i =
+      // D_{i-1} (A_0 = 0) at [0, nL), large slots ascending with their
+      // inclusive excess sums E_j at [nL, M) (both sequences sorted).
 #pragma unroll
       for (int j = 0; j < P; ++j) {
         const u64 a = static_cast<u64>(M) * q[j];
-        packed[j] = a < Qg ? (Qg - a) + (1ull << 48) : 0ull;
-      }
-      ptot = slot_scan_smem<C, u64>(packed, S.prob, G);
-#pragma unroll
-      for (int j = 0; j < P; ++j) pinc[j] = S.prob[C::slot(G.t, j)];
-    }
-    // (every thread read qinc before passing scan 2's barriers: S.scan is free)
-    const int nL = static_cast<int>(ptot >> 48);
-    const u64 Dtot = ptot & ((1ull << 48) - 1);
-    auto cls = [&](int j, bool& small, u64& a, u64& Dinc, u64& Einc, int& ls) {
-      a = static_cast<u64>(M) * q[j];
-      small = a < Qg;
-      Dinc = pinc[j] & ((1ull << 48) - 1);
-      ls = static_cast<int>(pinc[j] >> 48) - (small ? 1 : 0);   // smalls before the slot
-      const uint32_t slot1 = static_cast<uint32_t>(C::slot(G.t, j)) + 1u;
-      if constexpr (C::SCAN32) {   // Q < 2^32: 32 x 32 -> 64-bit products (one IMAD.WIDE each)
-        Einc = Dinc + static_cast<u64>(static_cast<uint32_t>(qinc[j])) * static_cast<uint32_t>(M) -
-               static_cast<u64>(slot1) * static_cast<uint32_t>(Qg);
-      } else {
-        Einc = Dinc + static_cast<u64>(M) * qinc[j] - static_cast<u64>(slot1) * Qg;
-      }
-    };
-    // Lists: small slots ascending with their EXCLUSIVE deficit sums A_i =
-    // D_{i-1} (A_0 = 0) at [0, nL), large slots ascending with their
-    // inclusive excess sums E_j at [nL, M) (both sequences sorted).
-#pragma unroll
-    for (int j = 0; j < P; ++j) {
-      bool small;
-      u64 a, Dinc, Einc;
-      int ls;
-      cls(j, small, a, Dinc, Einc, ls);
-      const int s = C::slot(G.t, j);
-      if (small) {
-        S.lists[ls] = s;
-        S.scan[ls] = Dinc - (Qg - a);
-      } else {
-        S.lists[nL + (s - ls)] = s;
-        S.scan[nL + (s - ls)] = Einc;
+        const bool small = a < Qg;
+        const u64 Dinc = pinc[j] & ((1ull << 48) - 1);
+        const int ls = static_cast<int>(pinc[j] >> 48) - (small ? 1 : 0);   // smalls before the slot
+        const int s = C::slot(G.t, j);
+        if (small) {
+          S.lists[ls] = s;
+          S.scan[ls] = Dinc - (Qg - a);
+        } else {   // E_s = D_s + sum_{s' <= s} (a_s' - Q)
+          S.lists[nL + (s - ls)] = s;
+          S.scan[nL + (s - ls)] = Dinc + static_cast<u64>(M) * qinc[j] - static_cast<u64>(s + 1) * Qg;
+        }
       }
     }
     gsync<C::GW>(G.g);
