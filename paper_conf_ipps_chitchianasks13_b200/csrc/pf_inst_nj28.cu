@@ -5,9 +5,11 @@
 #include "pf_registry.h"
 
 namespace pf {
+// (m = 256 without the split first load: C4's 16M-particle launches are
+// tens of rounds of sub-filters, where it measured +0.6 %)
 #define PF_LARGE_D_ENTRIES(NJ, RES, GW256, MINB256)                                                \
   PF_ENTRY(NJ, 32, RES, 1, 4, 1, 1, 1), PF_ENTRY(NJ, 64, RES, 2, 2, 1, 1, 1),                       \
-      PF_ENTRY(NJ, 128, RES, 4, 1, 1, 1, 1), PF_ENTRY(NJ, 256, RES, GW256, 1, 1, 1, MINB256),       \
+      PF_ENTRY(NJ, 128, RES, 4, 1, 1, 1, 1), PF_ENTRY_NOSPLIT(NJ, 256, RES, GW256, 1, 1, 1, MINB256), \
       PF_ENTRY(NJ, 512, RES, 16, 1, 1, 1, 1), PF_ENTRY(NJ, 1024, RES, 16, 1, 1, 1, 1)
 const KernelEntry kEntriesNJ28[] = {
     // m = 256 (config C4), measured: two particles per thread (packed f32x2 path with the

@@ -184,10 +184,15 @@ __device__ __forceinline__ unsigned long long tl_now() {
 #define PF_X2_DEFAULT 1
 #endif
 template <class Model_, int M_, int RES_, int GW_, int S_, int NSTAGE_, int UNR_, int MINB_, int EARLY_ = 0,
-          int X2_ = PF_X2_DEFAULT>
+          int X2_ = PF_X2_DEFAULT, int SPLIT0_ = 1>
 struct KCfg {
   using Model = Model_;
   static constexpr int EARLY = EARLY_;       // start the next TMA load right after the sample loop
+  // a group's first block in two bulk copies (log-weight row, then state
+  // rows): for mappings whose launch is a few rounds of sub-filters (the
+  // launch's first burst is a visible share of the step); the large-shard
+  // mappings (tens of rounds) measured +2.5 % with it and leave it out
+  static constexpr bool SPLIT0 = SPLIT0_ != 0;
   static constexpr int M = M_, RES = RES_, GW = GW_, S = S_, NSTAGE = NSTAGE_, UNR = UNR_;
   static constexpr int MINB = MINB_;         // __launch_bounds__ min CTAs per SM (register cap)
   static constexpr int D = Model::D;
@@ -217,8 +222,9 @@ struct KCfg {
   static constexpr size_t g_red = g_alias + ((RES == RES_VOSE && !PROB32) ? sizeof(int) * M : 0);   // u64 [2][32]
   static constexpr size_t g_cand = g_red + sizeof(u64) * 64;                     // u64 [GW KMAX + GW]
   static constexpr size_t g_misc = g_cand + sizeof(u64) * GW * (KMAX + 1);       // int [GW][2][KMAX]
-  static constexpr size_t g_bar = g_misc + sizeof(int) * GW * 2 * KMAX;          // u64 [2] + next [2]
-  static constexpr size_t group_bytes = (g_bar + 32 + 127) / 128 * 128;
+  // mbarriers: [2] log-weight row of stage 0/1, [2] state rows of stage 0/1; then next [2]
+  static constexpr size_t g_bar = g_misc + sizeof(int) * GW * 2 * KMAX;
+  static constexpr size_t group_bytes = (g_bar + 48 + 127) / 128 * 128;
   // per-CTA
   static constexpr size_t c_zin = 0;          // float [64]: z (ZD), h_s u (UD)
   static constexpr size_t c_zin2 = 256;       // f2 [64]: the same, each value duplicated (packed operands)
@@ -454,7 +460,7 @@ __device__ __forceinline__ void resample_group(const uint32_t (&q)[C::P], const 
       // weights (u32) and the packed deficits (u64) — one warp scan level and
       // one cross-warp level for the two — and writes its list entries
       // straight from registers (no scan results stored back to shared memory
-      // and re-read).  5 group barriers per table instead of 8; the same
+      // and re-read).  4 group barriers per table instead of 8; the same
       // sums, hence the same table.
       uint32_t qs = 0;
 #pragma unroll
@@ -1047,7 +1053,7 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
   S.alias = reinterpret_cast<int*>(gs + C::g_alias);
   S.lists = nullptr;   // per sub-filter: the stage's log-weight row
   uint2* bzw_s = reinterpret_cast<uint2*>(gs + C::g_scan);       // STAGED: Philox words after the resample
-  volatile unsigned int* next_s = reinterpret_cast<unsigned int*>(gs + C::g_bar + 16);
+  volatile unsigned int* next_s = reinterpret_cast<unsigned int*>(gs + C::g_bar + 32);
   GroupCtx G;
   G.g = g;
   G.t = threadIdx.x - g * C::T;
@@ -1072,13 +1078,33 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
   // finish early take more).  Thread 0 announces each next index through
   // next_s[barrier] before arriving on that barrier (release / acquire), and
   // a "no more work" index completes the barrier phase without a copy.
-  auto issue = [&](int b, long long nn) {   // thread 0 only
+  // A group's FIRST sub-filter arrives in two bulk copies: its log-weight
+  // row (row D of the block) on barrier b, and — requested only once that
+  // row has landed, so that every group's log-weights come first — its D
+  // state rows on barrier 2 + b.  The exchange selection, normalisation and
+  // resampler need only the log-weights, so at the launch's start — when
+  // every group's first block comes from HBM at once, ~18 MB at C2 — a group
+  // works on them while the state rows (9/10 of the bytes) are in flight.  Later sub-filters
+  // (their loads overlap the previous sub-filter's work, from L2 after the
+  // prefetch) come in one copy on barrier b; barrier 2 + b then completes at
+  // once.  (Splitting every load measured +3 % at 16M particles.)
+  const uint32_t lw_bytes = static_cast<uint32_t>(sizeof(float) * M);
+  const uint32_t st_bytes = stage_bytes - lw_bytes;
+  auto issue = [&](int b, long long nn, bool split) {   // thread 0 only
     next_s[b] = static_cast<unsigned int>(nn < P.n_local ? nn : P.n_local);
-    if (nn < P.n_local) {
-      mbar_arrive_expect_tx(bars + b, stage_bytes);
-      bulk_g2s(gs + C::g_stage + b * C::stage_bytes, P.parts + nn * ROW, stage_bytes, bars + b);
+    unsigned char* dst = gs + C::g_stage + b * C::stage_bytes;
+    const float* src = P.parts + nn * ROW;
+    if (C::SPLIT0 && nn < P.n_local && split) {   // (the state rows: issue_states)
+      mbar_arrive_expect_tx(bars + b, lw_bytes);
+      bulk_g2s(dst + st_bytes, src + static_cast<long long>(D) * M, lw_bytes, bars + b);
     } else {
-      mbar_arrive(bars + b);
+      if (nn < P.n_local) {
+        mbar_arrive_expect_tx(bars + b, stage_bytes);
+        bulk_g2s(dst, src, stage_bytes, bars + b);
+      } else {
+        mbar_arrive(bars + b);
+      }
+      if constexpr (C::SPLIT0) mbar_arrive(bars + 2 + b);
     }
   };
   // thread 0 keeps one dynamic index in flight: the atomic's latency is
@@ -1095,6 +1121,23 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
     return nn;
   };
 
+  // a6, the mailbox part: the K incoming entries of sub-filter gsf_ (offsets
+  // into woff, their log-weights in_w by lanes < K, this thread's first
+  // element of the copy into vpre)
+  auto mb_fetch = [&](long long gsf_, float& in_w_, float& vpre_) {
+    if (G.lane < K) {
+      const int qi = static_cast<int>((static_cast<uint32_t>(G.lane) * P.t_inv) >> 16);   // lane / t
+      const int off = static_cast<int>((neighbor_row(P, gsf_, qi) * P.tt + (G.lane - qi * P.t)) * E);
+      woff[G.lane] = off;
+      in_w_ = P.mb_prev[off];
+    }
+    __syncwarp();
+    if (G.t < K * E) {
+      const int j = G.t / E;
+      vpre_ = P.mb_prev[woff[j] + (G.t - j * E)];
+    }
+  };
+
   // programmatic dependent launch: the CTA's launch overlaps the previous
   // step's tail; nothing that step wrote (particle blocks, mailbox, counters,
   // key, device inputs) is read before its grid has completed (no-op otherwise)
@@ -1102,21 +1145,27 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
 #ifdef PF_TIMELINE
   const unsigned long long tl_pw = tl_now();
 #endif
+  // z / u first: their (device-input) loads leave before the launch's burst
+  // of first-sub-filter copies, not queued behind it
+  float zv = 0.0f, uv = 0.0f;
+  if (do_sample) {
+    if (threadIdx.x < ZD) zv = P.z ? P.z[threadIdx.x] : P.zin[threadIdx.x];
+    if (threadIdx.x < UD) uv = P.u ? P.u[threadIdx.x] : P.uin[threadIdx.x];
+  }
   if (G.t == 0) {
-    mbar_init(bars, 1);
-    mbar_init(bars + 1, 1);
+#pragma unroll
+    for (int b = 0; b < (C::SPLIT0 ? 4 : 2); ++b) mbar_init(bars + b, 1);
     fence_mbar_init();
-    issue(0, gid0);
+    issue(0, gid0, true);
     if (gid0 < P.n_local) pending = ticket_add(P.work);
   }
   if (do_sample) {
     if (threadIdx.x < ZD) {
-      const float v = P.z ? P.z[threadIdx.x] : P.zin[threadIdx.x];
-      z_s[threadIdx.x] = v;
-      z2_s[threadIdx.x] = bc(v);
+      z_s[threadIdx.x] = zv;
+      z2_s[threadIdx.x] = bc(zv);
     }
     if (threadIdx.x < UD) {   // control term h_s u_i (F8)
-      const float v = P.mc.hs * (P.u ? P.u[threadIdx.x] : P.uin[threadIdx.x]);
+      const float v = P.mc.hs * uv;
       hsu_s[threadIdx.x] = v;
       hsu2_s[threadIdx.x] = bc(v);
     }
@@ -1134,12 +1183,20 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
   for (int it = 0;; ++it) {
     const int st = (C::NSTAGE == 2) ? (it & 1) : 0;
     TL(tl_w0);
-    mbar_wait(bars + st, C::NSTAGE == 2 ? (it >> 1) & 1 : it & 1);
+    const uint32_t bpar = C::NSTAGE == 2 ? (it >> 1) & 1 : it & 1;
+    mbar_wait(bars + st, bpar);   // the log-weight row (and next_s)
+    if constexpr (C::SPLIT0) {   // first sub-filter: now its state rows
+      if (it == 0 && G.t == 0 && next_s[st] < P.n_local) {
+        const long long n0 = next_s[st];
+        mbar_arrive_expect_tx(bars + 2 + st, st_bytes);
+        bulk_g2s(gs + C::g_stage + st * C::stage_bytes, P.parts + n0 * ROW, st_bytes, bars + 2 + st);
+      }
+    }
     TL(tl_ready);
     const long long n = next_s[st];
     if (n >= P.n_local) break;
     if constexpr (C::NSTAGE == 2) {   // prefetch the next sub-filter into the other stage
-      if (G.t == 0) issue(st ^ 1, fetch_next());
+      if (G.t == 0) issue(st ^ 1, fetch_next(), false);
     }
     float* xs = reinterpret_cast<float*>(gs + C::g_stage + st * C::stage_bytes);
     float* ws = xs + D * M;
@@ -1152,7 +1209,7 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
       fence_proxy_async_smem();
       gsync<GW>(g);
       if constexpr (C::NSTAGE == 1) {
-        if (G.t == 0) issue(0, fetch_next());
+        if (G.t == 0) issue(0, fetch_next(), false);
       }
       issued = true;
     };
@@ -1168,6 +1225,18 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
 #pragma unroll
     for (int j = 0; j < PP; ++j) lw[j] = ws[C::slot(G.t, j)];
     uint32_t lmax_o = 0;   // ordered max of the post-exchange log-weights
+    bool defer_x = false;  // incoming state entry (this thread's vpre) not yet in the state rows
+    float dvx = 0.0f;
+    // the state rows: landed (bulk copy) + the deferred incoming entry, before the group barrier
+    // that precedes any read of them
+    auto states_in = [&]() {
+      if constexpr (!C::SPLIT0) return;
+      mbar_wait(bars + 2 + st, bpar);
+      if (defer_x && G.t < K * E) {
+        const int j = G.t / E, c = G.t - j * E;
+        if (c >= 2) xs[(c - 2) * M + wlist[j]] = dvx;
+      }
+    };
 
     // ---- a6 exchange: neighbours' best t (mailbox of step k-1) overwrite
     //      the own deg*t worst slots (R2–R5)
@@ -1190,17 +1259,7 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
       // and this thread's first element of the copy below (one L2 round trip
       // overlapped with the selection instead of two dependent ones).
       float in_w = 0.0f, vpre = 0.0f;
-      if (G.lane < K) {
-        const int qi = static_cast<int>((static_cast<uint32_t>(G.lane) * P.t_inv) >> 16);   // lane / t
-        const int off = static_cast<int>((neighbor_row(P, gsf, qi) * P.tt + (G.lane - qi * P.t)) * E);
-        woff[G.lane] = off;
-        in_w = P.mb_prev[off];
-      }
-      __syncwarp();
-      if (G.t < K * E) {
-        const int j = G.t / E;
-        vpre = P.mb_prev[woff[j] + (G.t - j * E)];
-      }
+      mb_fetch(gsf, in_w, vpre);
       u64 my_cand = ~0ull;
 #pragma unroll 1
       for (int j = 0; j < K; ++j) {
@@ -1257,14 +1316,21 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
         if ((s & (C::T - 1)) == G.t) excl |= 1u << (s / C::T);
       }
       const uint32_t in_max = __reduce_max_sync(0xFFFFFFFFu, G.lane < K ? ord_f32(in_w) : 0u);
+      // incoming log-weights now; incoming states into the state rows only
+      // once their bulk copy has landed: for the first (split) load deferred
+      // to after the resampler when every entry value is one thread's vpre
+      // (K E <= T), else waited for here (at once after an unsplit load)
+      defer_x = C::SPLIT0 && it == 0 && K * E <= C::T;
+      if (C::SPLIT0 && !defer_x) mbar_wait(bars + 2 + st, bpar);
 #pragma unroll 1
       for (int e = G.t; e < K * E; e += C::T) {
         const int j = e / E, c = e - j * E;
         const float v = e == G.t ? vpre : P.mb_prev[woff[j] + c];
         const int slot = wlist[j];
         if (c == 0) ws[slot] = v;
-        else if (c >= 2) xs[(c - 2) * M + slot] = v;
+        else if (c >= 2 && !defer_x) xs[(c - 2) * M + slot] = v;
       }
+      dvx = vpre;
       if (P.dbg_src) {
 #pragma unroll
         for (int i = 0; i < PP; ++i) {
@@ -1293,6 +1359,7 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
     }
 
     if (mode == MODE_EXCHANGE) {
+      states_in();   // (the copy must land before the stage is reused)
       finish();
       continue;
     }
@@ -1367,7 +1434,9 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
 #pragma unroll
         for (int j = 0; j < PP; ++j) P.dbg_anc[n * M + C::slot(G.t, j)] = anc[j];
       }
-      // all resampler reads of the scan buffer and the log-weight row are done
+      states_in();
+      // all resampler reads of the scan buffer and the log-weight row are done;
+      // the state rows are complete (bulk copy + incoming entries)
       gsync<GW>(g);
       if constexpr (C::STAGED) {
         // rolled sample loop: per-slot ancestor -> the (now free) log-weight

@@ -38,13 +38,15 @@ extern const KernelEntry kEntriesARMG[];   // the generic arm: n_joints key -NJM
 extern const int kNumEntriesARMG;
 }  // namespace pf
 
-// one table entry for model type MT (its kId, n_joints NJ)
-#define PF_ENTRY_MT(MT, NJ, LARGE, M, RES, GW, S, NST, UNR, MINB)                                     \
+// one table entry for model type MT (its kId, n_joints NJ); SPLIT = KCfg::SPLIT0
+#define PF_ENTRY_MTS(MT, NJ, LARGE, SPLIT, M, RES, GW, S, NST, UNR, MINB)                               \
   {MT::kId, NJ, M, RES, GW, S, NST, UNR, MINB, LARGE,                                               \
-   &StepKernel<KCfg<MT, M, RES, GW, S, NST, UNR, MINB>>::prepare,                                    \
-   &StepKernel<KCfg<MT, M, RES, GW, S, NST, UNR, MINB>>::launch,                                     \
-   &StepKernel<KCfg<MT, M, RES, GW, S, NST, UNR, MINB>>::resample_debug,                             \
-   StepKernel<KCfg<MT, M, RES, GW, S, NST, UNR, MINB>>::smem()}
+   &StepKernel<KCfg<MT, M, RES, GW, S, NST, UNR, MINB, 0, PF_X2_DEFAULT, SPLIT>>::prepare,           \
+   &StepKernel<KCfg<MT, M, RES, GW, S, NST, UNR, MINB, 0, PF_X2_DEFAULT, SPLIT>>::launch,            \
+   &StepKernel<KCfg<MT, M, RES, GW, S, NST, UNR, MINB, 0, PF_X2_DEFAULT, SPLIT>>::resample_debug,    \
+   StepKernel<KCfg<MT, M, RES, GW, S, NST, UNR, MINB, 0, PF_X2_DEFAULT, SPLIT>>::smem()}
+#define PF_ENTRY_MT(MT, NJ, LARGE, M, RES, GW, S, NST, UNR, MINB) \
+  PF_ENTRY_MTS(MT, NJ, LARGE, 1, M, RES, GW, S, NST, UNR, MINB)
 #define PF_ENTRY(NJ, M, RES, GW, S, NST, UNR, MINB) PF_ENTRY_MT(ArmPlanar<NJ>, NJ, 0, M, RES, GW, S, NST, UNR, MINB)
 // Default mapping for small states (d <= 12), measured on B200:
 // about four particles per thread (P = m / 32 GW), one warp per sub-filter up
@@ -58,4 +60,8 @@ extern const int kNumEntriesARMG;
 #define PF_LATENCY_ENTRIES(NJ, RES)                                                                  \
   PF_ENTRY(NJ, 64, RES, 2, 4, 1, 1, 3), PF_ENTRY(NJ, 128, RES, 4, 2, 1, 1, 3),                      \
       PF_ENTRY(NJ, 256, RES, 8, 1, 1, 1, 3)
-#define PF_ENTRY_LARGE(NJ, M, RES, GW, S, NST, UNR, MINB) PF_ENTRY_MT(ArmPlanar<NJ>, NJ, 1, M, RES, GW, S, NST, UNR, MINB)
+// large-shard mappings (tens of rounds of sub-filters per launch): no split first load (KCfg::SPLIT0)
+#define PF_ENTRY_LARGE(NJ, M, RES, GW, S, NST, UNR, MINB) \
+  PF_ENTRY_MTS(ArmPlanar<NJ>, NJ, 1, 0, M, RES, GW, S, NST, UNR, MINB)
+#define PF_ENTRY_NOSPLIT(NJ, M, RES, GW, S, NST, UNR, MINB) \
+  PF_ENTRY_MTS(ArmPlanar<NJ>, NJ, 0, 0, M, RES, GW, S, NST, UNR, MINB)

@@ -9,6 +9,7 @@ CONFIGS = [  # nj, m, N, resampler, topo, t
     (5, 256, 65536, "rws", "ring", 1), (5, 256, 65536, "vose", "ring", 1),
     (28, 256, 65536, "rws", "ring", 1), (28, 256, 65536, "vose", "ring", 1),
     (5, 256, 16384, "rws", "torus", 1), (5, 256, 16384, "rws", "ring", 0),
+    (5, 1048576, 1, "rws", "none", 0), (5, 1048576, 1, "vose", "none", 0),   # centralized filter (NEXT-2)
 ]
 
 
