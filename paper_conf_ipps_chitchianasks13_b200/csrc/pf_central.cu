@@ -3,15 +3,18 @@
 // reference scheme ("a sequential, centralized particle filter", PAPER.md:18
 // §VI; Fig.5 and Fig.9).  Same arithmetic contract, counter
 // layout and log-weight semantics as the distributed step (a1–a3, a5, a7–a10);
-// no exchange.  Three launches per step (k > 1):
+// no exchange.  RWS, two launches per step (k > 1):
 //   cz_tile_scan  q_i = expq(l_i - l_max) (l_max = the previous step's best,
 //                 from its estimate record) and per-tile inclusive u64 sums
-//   cz_tile_prefix  inclusive prefix of the tile totals (one CTA), Q
-//   cz_step       per particle: RWS draw (Philox (p, k, 0, 0) word 0, R9),
-//                 two-level binary search (tiles, then inside the tile),
-//                 gather from the previous buffer, sample + weight, store to
-//                 the other buffer, block argmax + u64 atomicMax; the last CTA
-//                 copies the winning particle to the estimate record.
+//                 (one CTA of 1024 threads per 4096-slot tile)
+//   cz_step       prologue: each CTA scans the tile totals into the tile
+//                 prefix in its shared memory (and Q; above 4M particles a
+//                 cz_tile_prefix launch does it instead); per particle: RWS
+//                 draw (Philox (p, k, 0, 0) word 0, R9), binary search (tiles
+//                 in shared memory, then inside the tile), gather from the
+//                 previous buffer, sample + weight, store to the other buffer,
+//                 block argmax + u64 atomicMax; the last CTA copies the
+//                 winning particle to the estimate record.
 // Particle buffers ping-pong: step k reads buffer (k-1)&1 and writes k&1.
 #include <cuda_runtime.h>
 
@@ -23,8 +26,8 @@
 namespace pf {
 namespace {
 
-constexpr int kScanThreads = 256;
-constexpr int kPerThread = kCentralTile / kScanThreads;   // 16 consecutive particles per thread
+constexpr int kScanThreads = 1024;
+constexpr int kPerThread = kCentralTile / kScanThreads;   // 4 consecutive particles per thread
 
 __device__ __forceinline__ u64 block_excl_scan(u64 v, u64* sm, u64& total) {
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
@@ -38,29 +41,46 @@ __device__ __forceinline__ u64 block_excl_scan(u64 v, u64* sm, u64& total) {
   return (warp > 0 ? off : 0ull) + x - v;
 }
 
+// The inclusive sums of one tile (one CTA of 1024 threads, 4 consecutive
+// slots per thread: a warp covers 128 slots, sum < 2^29, so the warp scan is
+// u32; the warp offsets are u64, tile < 2^34) and the tile total.
+__device__ __forceinline__ void tile_sums(const uint32_t (&q)[kPerThread], u64* __restrict__ cl,
+                                          u64* __restrict__ tile_sum) {
+  __shared__ uint32_t wtot[32];
+  __shared__ u64 woff_s[33];
+  const int t = threadIdx.x, lane = t & 31, warp = t >> 5;
+  uint32_t run[kPerThread];
+  uint32_t acc = 0;
+#pragma unroll
+  for (int j = 0; j < kPerThread; ++j) {
+    acc += q[j];
+    run[j] = acc;
+  }
+  const uint32_t x = warp_incl_scan<uint32_t>(acc, lane);
+  if (lane == 31) wtot[warp] = x;
+  __syncthreads();
+  if (warp == 0) {
+    const u64 wt = wtot[lane];
+    const u64 wi = warp_incl_scan<u64>(wt, lane);
+    woff_s[lane] = wi - wt;
+    if (lane == 31) woff_s[32] = wi;
+  }
+  __syncthreads();
+  const u64 off = woff_s[warp] + (x - acc);
+  ulonglong2* dst = reinterpret_cast<ulonglong2*>(cl + static_cast<long long>(blockIdx.x) * kCentralTile + t * kPerThread);
+  dst[0] = make_ulonglong2(off + run[0], off + run[1]);
+  dst[1] = make_ulonglong2(off + run[2], off + run[3]);
+  if (t == 0) tile_sum[blockIdx.x] = woff_s[32];
+}
+
 // a7: integer weights of one tile and their inclusive sums (u64).
 __global__ void __launch_bounds__(kScanThreads) cz_tile_scan(const float* __restrict__ logw, const float* record,
                                                              u64* __restrict__ cl, u64* __restrict__ tile_sum) {
-  __shared__ u64 sm[32];
   const float lmax = unord_f32(__float_as_uint(record[1]));   // ordered(l_max) is the key's high word
   const long long base = static_cast<long long>(blockIdx.x) * kCentralTile + threadIdx.x * kPerThread;
-  u64 run[kPerThread];
-  u64 acc = 0;
-#pragma unroll
-  for (int j = 0; j < kPerThread; j += 4) {
-    const float4 w4 = *reinterpret_cast<const float4*>(logw + base + j);
-    const float w[4] = {w4.x, w4.y, w4.z, w4.w};
-#pragma unroll
-    for (int e = 0; e < 4; ++e) {
-      acc += expq_c(w[e] - lmax);
-      run[j + e] = acc;
-    }
-  }
-  u64 total;
-  const u64 off = block_excl_scan(acc, sm, total);
-#pragma unroll
-  for (int j = 0; j < kPerThread; ++j) cl[base + j] = off + run[j];
-  if (threadIdx.x == 0) tile_sum[blockIdx.x] = total;
+  const float4 w4 = *reinterpret_cast<const float4*>(logw + base);
+  const uint32_t q[kPerThread] = {expq_c(w4.x - lmax), expq_c(w4.y - lmax), expq_c(w4.z - lmax), expq_c(w4.w - lmax)};
+  tile_sums(q, cl, tile_sum);
 }
 
 // Inclusive prefix of the tile totals (one CTA of 1024 threads).
@@ -454,22 +474,13 @@ __device__ __forceinline__ long long central_ancestor(const CentralParams& C, u6
 
 // Test hook: per-tile inclusive sums of given integer weights q (instead of
 // cz_tile_scan's q from the log-weights), then the ancestors for given uniforms.
-__global__ void __launch_bounds__(kScanThreads) cz_tile_scan_q(const uint32_t* __restrict__ q, u64* __restrict__ cl,
+__global__ void __launch_bounds__(kScanThreads) cz_tile_scan_q(const uint32_t* __restrict__ qin, u64* __restrict__ cl,
                                                                u64* __restrict__ tile_sum) {
-  __shared__ u64 sm[32];
   const long long base = static_cast<long long>(blockIdx.x) * kCentralTile + threadIdx.x * kPerThread;
-  u64 run[kPerThread];
-  u64 acc = 0;
+  uint32_t q[kPerThread];
 #pragma unroll
-  for (int j = 0; j < kPerThread; ++j) {
-    acc += q[base + j];
-    run[j] = acc;
-  }
-  u64 total;
-  const u64 off = block_excl_scan(acc, sm, total);
-#pragma unroll
-  for (int j = 0; j < kPerThread; ++j) cl[base + j] = off + run[j];
-  if (threadIdx.x == 0) tile_sum[blockIdx.x] = total;
+  for (int j = 0; j < kPerThread; ++j) q[j] = qin[base + j];
+  tile_sums(q, cl, tile_sum);
 }
 __global__ void __launch_bounds__(256) cz_draw_debug(const CentralParams C, const uint32_t* __restrict__ ua,
                                                      const uint32_t* __restrict__ ub, int* __restrict__ anc) {
@@ -502,11 +513,27 @@ __global__ void __launch_bounds__(256) cz_step(const CentralParams C) {
   const int tiles = static_cast<int>(M / kCentralTile);
   __shared__ u64 tidx_s[kTidxMax];   // RWS: the inclusive tile prefix
   const bool use_tidx = !C.vose && !C.first && !C.publish && tiles <= kTidxMax;
-  if (use_tidx)
-    for (int t = tid; t < tiles; t += blockDim.x) tidx_s[t] = C.tile_incl[t];
+  u64 Q = 0ull;
+  if (use_tidx) {   // the inclusive prefix of the tile totals (in place of a cz_tile_prefix launch)
+    const int per = (tiles + 255) / 256;   // <= 4 consecutive tiles per thread
+    u64 v[kTidxMax / 256], acc = 0;
+#pragma unroll
+    for (int j = 0; j < kTidxMax / 256; ++j) {
+      const int tt = tid * per + j;
+      v[j] = (j < per && tt < tiles) ? __ldg(C.tile_sum + tt) : 0ull;
+      acc += v[j];
+    }
+    u64 run = block_excl_scan(acc, red, Q);
+#pragma unroll
+    for (int j = 0; j < kTidxMax / 256; ++j) {
+      const int tt = tid * per + j;
+      run += v[j];
+      if (j < per && tt < tiles) tidx_s[tt] = run;
+    }
+  }
   const u64* tidx = use_tidx ? tidx_s : nullptr;
   __syncthreads();
-  const u64 Q = C.first ? 0ull : C.tile_incl[tiles - 1];
+  if (!use_tidx && !C.first) Q = C.tile_incl[tiles - 1];
   u64 best = 0ull;
   // one particle per thread (grid-stride): the gather from random ancestors
   // is latency-bound, so occupancy (registers) matters more than the packed
@@ -609,7 +636,8 @@ cudaError_t central_step_m(const CentralParams& c, int grid, cudaStream_t s) {
       vose_table(c, s);
     } else {
       cz_tile_scan<<<tiles, kScanThreads, 0, s>>>(logw, c.record_prev, c.cl, c.tile_sum);
-      cz_tile_prefix<<<1, 1024, 0, s>>>(c.tile_sum, c.tile_incl, tiles);
+      // the tile prefix: in every cz_step CTA's prologue when it fits its shared memory
+      if (tiles > kTidxMax) cz_tile_prefix<<<1, 1024, 0, s>>>(c.tile_sum, c.tile_incl, tiles);
     }
   }
   cz_step<Model><<<grid, 256, 0, s>>>(c);
