@@ -358,6 +358,16 @@ pf_status pf_peer_connect(pf_handle* h, const uint8_t* blobs);
 pf_status pf_peer_connect_local(pf_handle* const* handles, int32_t world);
 int32_t pf_peer_connected(const pf_handle* h);
 
+/* The step kernel's launch configuration chosen for this handle (tuning,
+ * tests; DESIGN.md §6 "mappings"): out = int32[8] { warps per group, groups
+ * per CTA, TMA stages, sample-loop unroll, min CTAs per SM (register cap),
+ * split first load (0/1), grid size in CTAs, number of compiled mappings for
+ * this (model, n_joints, m, resampler) — the range of the PF_VARIANT
+ * environment variable read by pf_init }.  Host only, no synchronisation.
+ * Errors: PF_EINVAL (NULL), PF_ESTATE (the centralized filter: its kernels
+ * have fixed shapes). */
+pf_status pf_query_mapping(const pf_handle* h, int32_t* out);
+
 /* Release host metadata; NULL-safe.  Does not free caller buffers. */
 pf_status pf_destroy(pf_handle* h);
 

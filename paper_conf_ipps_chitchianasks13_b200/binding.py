@@ -26,6 +26,7 @@ ENTRY_POINTS = [
     "pf_debug_resample", "pf_debug_exchange", "pf_set_trace", "pf_get_trace", "pf_destroy", "pf_strerror",
     "pf_last_error", "pf_supported", "pf_debug_math", "pf_debug_check_sqrt", "pf_estimate_mean", "pf_mean_partial",
     "pf_reduce_means", "pf_peer_export", "pf_peer_connect", "pf_peer_connect_local", "pf_peer_connected",
+    "pf_query_mapping",
 ]
 PF_MATH = {"sin": 0, "cos": 1, "log": 2, "expq": 3, "sqrt": 4, "sincos2pi": 5, "normal_pair": 6, "philox": 7}
 
@@ -95,6 +96,7 @@ def lib() -> C.CDLL:
             "pf_get_trace": [P, P, P],
             "pf_destroy": [P],
             "pf_last_error": [P],
+            "pf_query_mapping": [P, P],
         }
         for name, args in sig.items():
             fn = getattr(L, name)
@@ -284,6 +286,15 @@ def pf_peer_connect(h, blobs: bytes) -> None:
 def pf_peer_connect_local(handles) -> None:
     arr = (C.c_void_p * len(handles))(*[h.value for h in handles])
     check(lib().pf_peer_connect_local(arr, len(handles)), "pf_peer_connect_local")
+
+
+def pf_query_mapping(h) -> dict:
+    """The step kernel's launch configuration of handle h (include/pf.h pf_query_mapping)."""
+    out = (C.c_int32 * 8)()
+    check(lib().pf_query_mapping(h, out), "pf_query_mapping")
+    keys = ("warps_per_group", "groups_per_cta", "tma_stages", "unroll", "min_ctas_per_sm", "split_first_load",
+            "grid", "n_variants")
+    return dict(zip(keys, list(out)))
 
 
 def pf_peer_connected(h) -> bool:

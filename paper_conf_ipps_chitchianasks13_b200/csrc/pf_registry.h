@@ -19,6 +19,7 @@ struct KernelEntry {
   int model, nj, m, res;          // pf_model_id; n_joints (arm; -NJMAX = a generic bucket) or 1
   int gw, s, nstage, unr, minb;   // warps per group, groups per CTA, TMA stages, sample unroll, min CTAs/SM
   int large;                      // preferred when the shard has >= kLargeNLocal sub-filters
+  int split;                      // KCfg::SPLIT0: a group's first block in two bulk copies
   cudaError_t (*prepare)(int* blocks_per_sm);
   cudaError_t (*launch)(const StepParams& p, int grid, cudaStream_t s, bool pdl);
   cudaError_t (*resample_debug)(const uint32_t* q, const uint32_t* ua, const uint32_t* ub, int* anc,
@@ -40,7 +41,7 @@ extern const int kNumEntriesARMG;
 
 // one table entry for model type MT (its kId, n_joints NJ); SPLIT = KCfg::SPLIT0
 #define PF_ENTRY_MTS(MT, NJ, LARGE, SPLIT, M, RES, GW, S, NST, UNR, MINB)                               \
-  {MT::kId, NJ, M, RES, GW, S, NST, UNR, MINB, LARGE,                                               \
+  {MT::kId, NJ, M, RES, GW, S, NST, UNR, MINB, LARGE, SPLIT,                                        \
    &StepKernel<KCfg<MT, M, RES, GW, S, NST, UNR, MINB, 0, PF_X2_DEFAULT, SPLIT>>::prepare,           \
    &StepKernel<KCfg<MT, M, RES, GW, S, NST, UNR, MINB, 0, PF_X2_DEFAULT, SPLIT>>::launch,            \
    &StepKernel<KCfg<MT, M, RES, GW, S, NST, UNR, MINB, 0, PF_X2_DEFAULT, SPLIT>>::resample_debug,    \

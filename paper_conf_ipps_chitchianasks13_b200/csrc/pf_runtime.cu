@@ -1184,6 +1184,21 @@ pf_status pf_peer_connect_local(pf_handle* const* handles, int32_t world) {
 
 int32_t pf_peer_connected(const pf_handle* h) { return h && h->peers ? 1 : 0; }
 
+pf_status pf_query_mapping(const pf_handle* h, int32_t* out) {
+  if (!h || !out) return PF_EINVAL;
+  if (h->g.central || !h->ke) return PF_ESTATE;
+  const pf::KernelEntry& e = *h->ke;
+  int n = 0;   // compiled mappings of (model, n_joints, m, resampler): the range of PF_VARIANT
+  for (int ti = 0; ti < kTables; ++ti) {
+    const Table t = tables(ti);
+    for (int i = 0; i < t.n; ++i)
+      if (matches(t.e[i], h->g.model, h->g.nj, h->g.m, h->cfg.resampler)) ++n;
+  }
+  const int32_t v[8] = {e.gw, e.s, e.nstage, e.unr, e.minb, e.split, h->grid, n};
+  std::memcpy(out, v, sizeof(v));
+  return PF_OK;
+}
+
 pf_status pf_destroy(pf_handle* h) {
   if (!h) return PF_OK;
   cudaStreamSynchronize(h->stream);
