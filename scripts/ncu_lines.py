@@ -19,4 +19,4 @@ for r in csv.reader(out.splitlines()):
 agg.sort(reverse=True)
 print(f"total warp-inst {tot_i}  stall samples {tot_s}")
 for ie, ss, f, ln, src in agg[:top]:
-    print(f"{100*ie/tot_i:5.1f}% {100*ss/max(tot_s,1):5.1f}%  {f}:{ln:<4} {src}")
+    print(f"{100*ie/tot_i:5.1f}% {100*ss/max(tot_s,1):5.1f}%  {f}:{ln:<4} {src}  [{ie} {ss}]")
