@@ -83,6 +83,8 @@ def test_query_mapping_defaults(P, W):
         return mp
     c2 = mapping(4096)
     assert (c2["warps_per_group"], c2["groups_per_cta"], c2["min_ctas_per_sm"], c2["split_first_load"]) == (2, 4, 3, 1)
+    c2v = mapping(4096, "vose")
+    assert (c2v["warps_per_group"], c2v["groups_per_cta"], c2v["min_ctas_per_sm"]) == (2, 4, 3)
     big = mapping(65536)
     assert (big["warps_per_group"], big["groups_per_cta"], big["min_ctas_per_sm"], big["split_first_load"]) == (2, 4, 4, 0)
     bigv = mapping(65536, "vose")
