@@ -6,12 +6,15 @@ runs in libpf_b200.so; this class only marshals arguments (binding.py).
 """
 from __future__ import annotations
 
+import ctypes
 from dataclasses import dataclass
 
 import numpy as np
 import torch
 
 from . import binding as B
+
+_cchar, _addressof = ctypes.c_char, ctypes.addressof
 
 TOPO = {"none": B.PF_TOPO_NONE, "ring": B.PF_TOPO_RING, "torus": B.PF_TOPO_TORUS2D, "all2all": B.PF_TOPO_ALL2ALL}
 RESAMPLER = {"rws": B.PF_RESAMPLE_RWS, "vose": B.PF_RESAMPLE_VOSE}
@@ -182,7 +185,12 @@ class ParticleFilter:
         else:   # copied into the launch by pf_step (host inputs travel with the kernel)
             if (type(z) is np.ndarray and type(u) is np.ndarray and z.dtype == np.float32 and u.dtype == np.float32
                     and z.flags.c_contiguous and u.flags.c_contiguous and z.size == self.zd and u.size == self.ud):
-                st = self._step_fn(self.h, z.ctypes.data, u.ctypes.data)   # no staging copy
+                # no staging copy; the address through the buffer protocol (writable
+                # arrays) costs a third of ndarray.ctypes.data, which builds an object
+                zf, uf = z.flags, u.flags
+                zp = _addressof(_cchar.from_buffer(z)) if zf.writeable else z.ctypes.data
+                up = _addressof(_cchar.from_buffer(u)) if uf.writeable else u.ctypes.data
+                st = self._step_fn(self.h, zp, up)
             else:
                 np.copyto(self._zin, z, casting="same_kind")
                 np.copyto(self._uin, u, casting="same_kind")
