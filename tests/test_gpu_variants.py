@@ -91,3 +91,16 @@ def test_query_mapping_defaults(P, W):
     assert (bigv["groups_per_cta"], bigv["min_ctas_per_sm"], bigv["split_first_load"]) == (7, 2, 0)
     small = mapping(16)
     assert small["warps_per_group"] == 8
+
+
+def test_query_mapping_errors(P, W):
+    # include/pf.h: NULL -> PF_EINVAL; the centralized filter (fixed kernel shapes) -> PF_ESTATE
+    import ctypes as C
+    from paper_conf_ipps_chitchianasks13_b200 import binding as B
+    tr = W.make_trajectory(5, 3, 0)
+    g = P.ParticleFilter(tr["mu0"], tr["sigma0"], P.ArmModel(n_joints=5), m=8192, n_filters=1, t=0, topo="none")
+    out = (C.c_int32 * 8)()
+    assert B.lib().pf_query_mapping(g.h, out) == B.PF_ESTATE
+    assert B.lib().pf_query_mapping(g.h, None) == B.PF_EINVAL
+    assert B.lib().pf_query_mapping(None, out) == B.PF_EINVAL
+    g.close()
