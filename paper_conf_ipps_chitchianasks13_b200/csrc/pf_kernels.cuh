@@ -1260,52 +1260,98 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
       // overlapped with the selection instead of two dependent ones).
       float in_w = 0.0f, vpre = 0.0f;
       mb_fetch(gsf, in_w, vpre);
-      u64 my_cand = ~0ull;
-#pragma unroll 1
-      for (int j = 0; j < K; ++j) {
-        u64 mk = key[0];
+      if (K == 2) {
+        // deg t = 2 (ring, t = 1: the benchmark configurations): each thread's
+        // two smallest keys, two warp rounds (the owner of the first advances
+        // to its second), then the group's two smallest of the GW sorted pairs
+        // — the same worst two (keys are unique), in the same order, without
+        // the K-round rescans and clears over every key
+        u64 m1 = ~0ull, m2 = ~0ull;
 #pragma unroll
-        for (int i = 1; i < PP; ++i) mk = key[i] < mk ? key[i] : mk;
-        const u64 wk = warp_min_u64(mk);
+        for (int i = 0; i < PP; ++i) {
+          const u64 kk = key[i];
+          const bool lt1 = kk < m1;
+          m2 = lt1 ? m1 : (kk < m2 ? kk : m2);
+          m1 = lt1 ? kk : m1;
+        }
+        const u64 w1 = warp_min_u64(m1);
+        if (m1 == w1) m1 = m2;
+        const u64 w2 = warp_min_u64(m1);
+        u64 b1 = w1, b2 = w2;
+        if constexpr (GW == 1) {
+          lmax_o = wmax;
+        } else {
+          if (G.lane == 0) {
+            cand[G.wig * 2] = w1;
+            cand[G.wig * 2 + 1] = w2;
+            cand[GW * C::KMAX + G.wig] = wmax;
+          }
+          gsync<GW>(g);
+          uint32_t mo = 0;
+          b1 = ~0ull;
+          b2 = ~0ull;
 #pragma unroll
-        for (int i = 0; i < PP; ++i)
-          if (key[i] == wk) key[i] = ~0ull;   // keys are unique (slot in the low bits)
-        if (G.lane == j) my_cand = wk;
-      }
-      if constexpr (GW == 1) {
-        lmax_o = wmax;
-        if (G.lane < K) wlist[G.lane] = static_cast<int>(0xFFFFFFFFu - static_cast<uint32_t>(my_cand));
+          for (int ww = 0; ww < GW; ++ww) {
+            mo = max(mo, static_cast<uint32_t>(cand[GW * C::KMAX + ww]));
+            const u64 x1 = cand[2 * ww], x2 = cand[2 * ww + 1];   // x1 < x2
+            if (x1 < b1) {
+              b2 = b1 < x2 ? b1 : x2;
+              b1 = x1;
+            } else {
+              b2 = b2 < x1 ? b2 : x1;
+            }
+          }
+          lmax_o = mo;
+        }
+        if (G.lane < 2) wlist[G.lane] = static_cast<int>(0xFFFFFFFFu - static_cast<uint32_t>(G.lane == 0 ? b1 : b2));
       } else {
-        // flat list: candidate i of the GW * K is cand[i] (warp i / K), the
-        // per-warp maxima after the GW * KMAX candidate slots
-        if (G.lane < K) cand[G.wig * K + G.lane] = my_cand;
-        if (G.lane == 0) cand[GW * C::KMAX + G.wig] = wmax;
-        gsync<GW>(g);
-        // every warp merges the GW candidate lists (identical result in all warps)
-        u64 c[GW];   // candidate i = lane + 32 r of the GW*K list
-        const int ncand = GW * K;
-#pragma unroll
-        for (int r = 0; r < GW; ++r) {
-          const int i = G.lane + 32 * r;
-          c[r] = i < ncand ? cand[i] : ~0ull;
-        }
-        uint32_t mo = 0;
-#pragma unroll
-        for (int ww = 0; ww < GW; ++ww) mo = max(mo, static_cast<uint32_t>(cand[GW * C::KMAX + ww]));
-        lmax_o = mo;
-        u64 mine = ~0ull;
-#pragma unroll 1
+        u64 my_cand = ~0ull;
+  #pragma unroll 1
         for (int j = 0; j < K; ++j) {
-          u64 lo = ~0ull;
-#pragma unroll
-          for (int r = 0; r < GW; ++r) lo = c[r] < lo ? c[r] : lo;
-          const u64 wk = warp_min_u64(lo);
-#pragma unroll
-          for (int r = 0; r < GW; ++r)
-            if (c[r] == wk) c[r] = ~0ull;
-          if (G.lane == j) mine = wk;
+          u64 mk = key[0];
+  #pragma unroll
+          for (int i = 1; i < PP; ++i) mk = key[i] < mk ? key[i] : mk;
+          const u64 wk = warp_min_u64(mk);
+  #pragma unroll
+          for (int i = 0; i < PP; ++i)
+            if (key[i] == wk) key[i] = ~0ull;   // keys are unique (slot in the low bits)
+          if (G.lane == j) my_cand = wk;
         }
-        if (G.lane < K) wlist[G.lane] = static_cast<int>(0xFFFFFFFFu - static_cast<uint32_t>(mine));
+        if constexpr (GW == 1) {
+          lmax_o = wmax;
+          if (G.lane < K) wlist[G.lane] = static_cast<int>(0xFFFFFFFFu - static_cast<uint32_t>(my_cand));
+        } else {
+          // flat list: candidate i of the GW * K is cand[i] (warp i / K), the
+          // per-warp maxima after the GW * KMAX candidate slots
+          if (G.lane < K) cand[G.wig * K + G.lane] = my_cand;
+          if (G.lane == 0) cand[GW * C::KMAX + G.wig] = wmax;
+          gsync<GW>(g);
+          // every warp merges the GW candidate lists (identical result in all warps)
+          u64 c[GW];   // candidate i = lane + 32 r of the GW*K list
+          const int ncand = GW * K;
+  #pragma unroll
+          for (int r = 0; r < GW; ++r) {
+            const int i = G.lane + 32 * r;
+            c[r] = i < ncand ? cand[i] : ~0ull;
+          }
+          uint32_t mo = 0;
+  #pragma unroll
+          for (int ww = 0; ww < GW; ++ww) mo = max(mo, static_cast<uint32_t>(cand[GW * C::KMAX + ww]));
+          lmax_o = mo;
+          u64 mine = ~0ull;
+  #pragma unroll 1
+          for (int j = 0; j < K; ++j) {
+            u64 lo = ~0ull;
+  #pragma unroll
+            for (int r = 0; r < GW; ++r) lo = c[r] < lo ? c[r] : lo;
+            const u64 wk = warp_min_u64(lo);
+  #pragma unroll
+            for (int r = 0; r < GW; ++r)
+              if (c[r] == wk) c[r] = ~0ull;
+            if (G.lane == j) mine = wk;
+          }
+          if (G.lane < K) wlist[G.lane] = static_cast<int>(0xFFFFFFFFu - static_cast<uint32_t>(mine));
+        }
       }
       __syncwarp();
       // own slots among the worst K (slot s is owned by thread s mod T, index s / T)
