@@ -1260,6 +1260,7 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
       // overlapped with the selection instead of two dependent ones).
       float in_w = 0.0f, vpre = 0.0f;
       mb_fetch(gsf, in_w, vpre);
+      int ws0 = 0, ws1 = 0;   // K = 2: the two worst slots, in every thread's registers
       if (K == 2) {
         // deg t = 2 (ring, t = 1: the benchmark configurations): each thread's
         // two smallest keys, two warp rounds (the owner of the first advances
@@ -1303,7 +1304,9 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
           }
           lmax_o = mo;
         }
-        if (G.lane < 2) wlist[G.lane] = static_cast<int>(0xFFFFFFFFu - static_cast<uint32_t>(G.lane == 0 ? b1 : b2));
+        ws0 = static_cast<int>(0xFFFFFFFFu - static_cast<uint32_t>(b1));
+        ws1 = static_cast<int>(0xFFFFFFFFu - static_cast<uint32_t>(b2));
+        if (G.lane < 2) wlist[G.lane] = G.lane == 0 ? ws0 : ws1;   // (states_in, the trace hook)
       } else {
         u64 my_cand = ~0ull;
   #pragma unroll 1
@@ -1356,10 +1359,15 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
       __syncwarp();
       // own slots among the worst K (slot s is owned by thread s mod T, index s / T)
       uint32_t excl = 0;
+      if (K == 2) {
+        excl = ((ws0 & (C::T - 1)) == G.t ? 1u << (ws0 / C::T) : 0u) |
+               ((ws1 & (C::T - 1)) == G.t ? 1u << (ws1 / C::T) : 0u);
+      } else {
 #pragma unroll 1
-      for (int j = 0; j < K; ++j) {
-        const int s = wlist[j];
-        if ((s & (C::T - 1)) == G.t) excl |= 1u << (s / C::T);
+        for (int j = 0; j < K; ++j) {
+          const int s = wlist[j];
+          if ((s & (C::T - 1)) == G.t) excl |= 1u << (s / C::T);
+        }
       }
       const uint32_t in_max = __reduce_max_sync(0xFFFFFFFFu, G.lane < K ? ord_f32(in_w) : 0u);
       // incoming log-weights now; incoming states into the state rows only
@@ -1372,7 +1380,7 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
       for (int e = G.t; e < K * E; e += C::T) {
         const int j = e / E, c = e - j * E;
         const float v = e == G.t ? vpre : P.mb_prev[woff[j] + c];
-        const int slot = wlist[j];
+        const int slot = K == 2 ? (j == 0 ? ws0 : ws1) : wlist[j];
         if (c == 0) ws[slot] = v;
         else if (c >= 2 && !defer_x) xs[(c - 2) * M + slot] = v;
       }
