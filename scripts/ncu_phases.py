@@ -2,15 +2,40 @@
 (scripts/ncu_lines.py report N output, every line): executed warp-instructions -> lane-instructions per
 particle and stall samples, grouped by the phase each CUDA source line belongs to.
 usage: ncu_phases.py lines.txt particles"""
-import re, sys
+import os, re, sys
 src, particles = sys.argv[1], int(sys.argv[2])
-K = {  # pf_kernels.cuh line ranges (this revision) -> phase
-    "exchange (a6)": [(672, 698), (1241, 1367)],
-    "normalise + resample (a7, a8)": [(348, 671), (1368, 1470)],
-    "sample loop glue: gather, stores (a9, a10)": [(699, 876), (1471, 1583)],
-    "local reduce + global key (a4, a5)": [(1584, 1668)],
-    "epilogue: last CTA, peers (a5)": [(877, 1023), (1669, 99999)],
-    "group helpers (barriers, warp reductions, slot / smem addressing), scheduling, TMA": [(1, 347), (1024, 1240)],
+# pf_kernels.cuh line ranges -> phase, found from the section markers of the source file itself
+KSRC = open(os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))),
+                         "paper_conf_ipps_chitchianasks13_b200", "csrc", "pf_kernels.cuh")).read().split("\n")
+
+
+def _at(pat, start=0):
+    for i in range(start, len(KSRC)):
+        if pat in KSRC[i]:
+            return i + 1   # 1-based line number
+    raise SystemExit(f"marker not found: {pat}")
+
+
+_scan = _at("X slot_scan_smem(") - 1
+_nbr = _at("long long neighbor_row(")
+_noise = _at("struct NoiseGen {")
+_peer = _at("static __device__ void peer_halo_rows(")
+_kern = _at(") pf_step_kernel(")
+_mbf0 = _at("auto mb_fetch = ", _kern)
+_mbf1 = _at("  };", _mbf0)
+_a6 = _at("// ---- a6 exchange", _kern)
+_a7 = _at("// ---- a7 normalise", _a6)
+_a9 = _at("// ---- a9 gather", _a7)
+_a4 = _at("// ---- a4 local reduce", _a9)
+_a5 = _at("// ---- a5: the last CTA", _a4)
+_end = _at("pf_resample_debug_kernel(", _a5)
+K = {
+    "exchange (a6)": [(_nbr, _noise - 1), (_mbf0, _mbf1), (_a6, _a7 - 1)],
+    "normalise + resample (a7, a8)": [(_scan, _nbr - 1), (_a7, _a9 - 1)],
+    "sample loop glue: gather, stores (a9, a10)": [(_noise, _peer - 1), (_a9, _a4 - 1)],
+    "local reduce + global key (a4, a5)": [(_a4, _a5 - 1)],
+    "epilogue: last CTA, peers (a5)": [(_peer, _kern - 1), (_a5, _end)],
+    "group helpers (barriers, warp reductions, slot / smem addressing), scheduling, TMA": [(1, _scan - 1), (_kern, _a6 - 1)],
 }
 D = {  # pf_device.cuh line ranges -> contract part
     "Philox4x32-10 (R12, F1)": [(23, 67)],
