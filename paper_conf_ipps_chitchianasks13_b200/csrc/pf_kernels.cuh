@@ -1658,17 +1658,14 @@ __global__ void __launch_bounds__(C::T* C::S, C::MINB) pf_step_kernel(const __gr
           nb_l = static_cast<u64>(n * P.tt + jb);
         }
         const int bslot = static_cast<int>(0xFFFFFFFFu - static_cast<uint32_t>(best) - pbase);
-#pragma unroll
-        for (int j = 0; j < PP; ++j) {
-          if (C::slot(G.t, j) == bslot) {   // unique owner
-            done |= 1u << j;
-            if (jb < P.t) {
-              float* e = P.mb_cur + (n * P.tt + jb) * E;
-              e[0] = lnew[j];
-              e[1] = __uint_as_float(pbase + bslot);
-            }
-            if (jb == 0) atomicMax(P.key_cur, best);
+        if ((bslot & (C::T - 1)) == G.t) {   // the unique owner (slot bslot = j T + t)
+          done |= 1u << (bslot / C::T);
+          if (jb < P.t) {
+            float* e = P.mb_cur + (n * P.tt + jb) * E;
+            e[0] = unord_f32(static_cast<uint32_t>(best >> 32));   // = lnew[j] (ord is a bijection)
+            e[1] = __uint_as_float(pbase + bslot);
           }
+          if (jb == 0) atomicMax(P.key_cur, best);
         }
         if (jb < P.t && G.wig == 0) {
           // the state of the best particle, one component per lane (one L2
