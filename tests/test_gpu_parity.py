@@ -140,6 +140,10 @@ def test_full_filter_c1(P, orc, W):
     # best t into their running pool candidates (All-to-All, t >= 2)
     (5, 32, 8192, 2, "all2all", "rws"),
     (5, 32, 8192, 4, "all2all", "vose"),
+    # deg t = 2 and 4 with four slots per thread (the specialised worst-slot selections)
+    (5, 256, 2048, 2, "ring", "rws"),
+    (5, 256, 1024, 1, "torus", "vose"),
+    (5, 256, 1024, 1, "ring", "rws"),
 ])
 def test_full_filter_variants(P, orc, W, nj, m, N, t, topo, res):
     _run_compare(P, orc, W, nj, m, N, 12, t=t, topo=topo, res=res, seed=nj * 1000 + m)
